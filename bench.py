@@ -1,0 +1,390 @@
+#!/usr/bin/env python
+"""Benchmark of the fused pointing->map hot path (BASELINE.json metric) on N B200s.
+
+One step = zero the map + toast_pointing_to_map over one observation (all of SURVEY 8(a)
+A1-A4 in one kernel) + (N > 1) one NCCL all-reduce of the map.  Weak scaling: every rank
+processes its own observation of the configured workload (TOAST distributes observations
+over processes) and the partial maps are summed.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c2] [--impl ours|reference]
+
+Prints ONE JSON line on rank 0.  `--impl reference` times the CPU oracle (OpenMP timing
+mode) on a bounded sample of the same workload, on rank 0 only.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "detector-samples/sec pointing→map (fused) at 1/2/4/8 B200; % of HBM/fp64 roofline"
+UNIT = "det-samples/s"
+
+# Algorithmic fp64 work per det-sample (FMA = 2 flops): quaternion
+# product 28, dir 13, orient 10, bx/by 13, cos/sin 2psi 15, HWP rotation 6, eta*cal 2,
+# HEALPix ~10 + atan2 30 + 1/3 sqrt 6, noise weighting 4  ->  ~133.
+F_ALG = 133.0
+SMS = 148
+DFMA_PER_SM_PER_CLK = 64  # B200 fp64 pipe
+
+WORKLOAD_DESC = {
+    "c1": "tiny satellite scan: 4 dets x 100k samples, nside 64 RING, IQU, no HWP",
+    "c2": "small ground scan: 64 dets x 1M samples, nside 256 NESTED, HWP + flags",
+    "c3": "medium ground scan: 1024 dets x 60k samples, nside 1024, IQU",
+    "c4": "large satellite: 2048 dets x 3.2M samples (1 day @ 37 Hz), nside 2048 NESTED",
+    "c5": "TOAST-benchmark-shaped observation: 2048 dets x 133200 samples, 60 intervals, nside 4096 NESTED",
+}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--workload", default="c2", choices=sorted(WORKLOAD_DESC))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--soak", type=float, default=1.0, help="seconds of untimed steps before timing (clocks)")
+    return ap.parse_args()
+
+
+# ----------------------------------------------------------------------------- clocks
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled every 100 ms (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.path = None
+
+    def start(self):
+        fd, self.path = tempfile.mkstemp(suffix=".csv")
+        os.close(fd)
+        q = ("timestamp,index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except (FileNotFoundError, OSError):
+            self.proc = None
+        self.t0 = time.time()
+
+    def stop(self):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self, t_start: float, t_end: float):
+        if self.proc is None or not self.path:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        rows = []
+        for line in open(self.path):
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) < 10:
+                continue
+            try:
+                ts = time.mktime(time.strptime(parts[0].split(".")[0], "%Y/%m/%d %H:%M:%S"))
+                rows.append((ts, float(parts[2]), float(parts[3]), parts[6:10]))
+            except ValueError:
+                continue
+        os.unlink(self.path)
+        win = [r for r in rows if t_start - 1.0 <= r[0] <= t_end + 1.0]
+        if len(win) < 3:
+            win = rows
+        if not win:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in win for i, v in enumerate(r[3]) if v.lower() == "active"})
+        return {"sm_mhz": statistics.median(r[1] for r in win), "sm_max_mhz": max(r[2] for r in win),
+                "reasons": reasons, "samples": len(win)}
+
+
+# ----------------------------------------------------------------------------- dist
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def algorithmic_bytes(w, det_samples: int) -> float:
+    """HBM bytes one step must move: TOD + det flags per det-sample,
+    boresight/HWP/shared flags per sample, one zeroing write + one write-back of the map."""
+    n_in = det_samples // w.n_det
+    b = det_samples * (8 + (1 if w.det_flags is not None else 0))
+    b += n_in * (32 + (8 if w.hwp is not None else 0) + (1 if w.shared_flags is not None else 0))
+    b += 2 * w.npix * w.nnz * 8
+    return float(b)
+
+
+# ----------------------------------------------------------------------------- cpu baseline
+
+def cpu_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count() or 1
+
+
+def cpu_sample_workload(name: str, target_det_samples: float, obs: int = 0):
+    """A bounded sample of the workload: all detectors of the first samples of the observation."""
+    from paper_conf_sc_demeurekktbb23_b200 import synth
+    full = synth.CONFIGS[name]
+    n_det, n_samp = full[1], full[2]
+    ns = int(min(n_samp, max(1000, target_det_samples / n_det)))
+    w = synth.make_workload(name, n_samp=ns, obs=obs)
+    return w
+
+
+def time_oracle(w, threads: int):
+    import oracle
+    zmap = np.zeros((w.n_submap, w.n_pix_submap, w.nnz))
+    t0 = time.perf_counter()
+    used = oracle.pointing_to_map_omp(w.fp_quats, w.boresight, w.epsilon, w.cal, w.det_scale, w.det_data, w.intervals,
+                                      w.nside, w.nest, w.nnz, w.global2local, w.n_pix_submap, zmap, hwp=w.hwp,
+                                      det_flags=w.det_flags, det_flag_mask=w.det_flag_mask,
+                                      shared_flags=w.shared_flags, shared_flag_mask=w.shared_flag_mask,
+                                      n_threads=threads)
+    return time.perf_counter() - t0, used
+
+
+def cpu_baseline(name: str, seconds_target: float = 15.0):
+    cores = cpu_cores()
+    probe = cpu_sample_workload(name, 2e6)
+    dt, used = time_oracle(probe, cores)
+    rate = probe.det_samples / max(dt, 1e-9)
+    w = cpu_sample_workload(name, rate * seconds_target)
+    dt, used = time_oracle(w, cores)
+    return {"value": w.det_samples / dt, "unit": UNIT, "cores": used, "kind": "oracle",
+            "sample": f"{w.n_det} dets x first {w.n_samp} samples of observation 0 ({w.det_samples} det-samples), "
+                      f"oracle OpenMP timing mode (omp atomic map updates), {dt:.1f} s"}
+
+
+def run_reference(args):
+    world, rank, local = dist_env()
+    if rank != 0:
+        return
+    cores = cpu_cores()
+    probe = cpu_sample_workload(args.workload, 1e6)
+    dt, used = time_oracle(probe, cores)
+    rate = probe.det_samples / max(dt, 1e-9)
+    # each step: a sample sized to ~1.5 s so the whole run stays within a few minutes
+    w = cpu_sample_workload(args.workload, rate * 1.5)
+    for _ in range(args.warmup):
+        time_oracle(w, cores)
+    times = []
+    for _ in range(args.steps):
+        dt, used = time_oracle(w, cores)
+        times.append(dt)
+    tot = sum(times)
+    value = w.det_samples * args.steps / tot
+    sample = (f"per step {w.n_det} dets x first {w.n_samp} samples ({w.det_samples} det-samples) of "
+              f"{args.workload}, oracle OpenMP timing mode")
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"{args.workload}: {WORKLOAD_DESC[args.workload]}", "oracle_sample": sample},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": used, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------------------- ours
+
+def main():
+    args = parse()
+    world, rank, local = dist_env()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_demeurekktbb23_b200 import binding, synth
+    from paper_conf_sc_demeurekktbb23_b200.staging import DeviceWorkload
+
+    if not torch.cuda.is_available():
+        raise SystemExit("bench.py needs a CUDA device (there is no CPU fallback)")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    binding.load()
+
+    w = synth.make_workload(args.workload, obs=rank)
+    dw = DeviceWorkload.upload(w, "cuda")
+    det_samples = w.det_samples
+    stream = torch.cuda.current_stream()
+    raw = dw.raw_args(stream)
+    lib = binding.load()
+    call = lib.toast_pointing_to_map
+
+    def step(k0=None, k1=None):
+        dw.zmap.zero_()
+        if k0 is not None:
+            k0.record(stream)
+        rc = call(*raw)
+        if rc != 0:
+            raise binding.ToastError(lib.toast_last_error().decode())
+        if k1 is not None:
+            k1.record(stream)
+        if world > 1:
+            dist.all_reduce(dw.zmap, op=dist.ReduceOp.SUM)
+
+    for _ in range(max(3, args.warmup)):
+        step()
+    torch.cuda.synchronize()
+    # soak: keep the GPU busy so clocks settle before the timed region
+    t_end_soak = time.time() + args.soak
+    while time.time() < t_end_soak:
+        for _ in range(20):
+            step()
+        torch.cuda.synchronize()
+
+    sampler = ClockSampler(local)
+    sampler.start()
+    time.sleep(0.3)
+    k_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t_wall0 = time.time()
+    e0.record(stream)
+    for i in range(args.steps):
+        step(*k_ev[i])
+    e1.record(stream)
+    torch.cuda.synchronize()
+    t_wall1 = time.time()
+    if world > 1:
+        dist.barrier()
+    ms = e0.elapsed_time(e1)
+    kern_ms = statistics.mean(a.elapsed_time(b) for a, b in k_ev)
+    time.sleep(0.2)
+    sampler.stop()
+    clocks = sampler.summary(t_wall0, t_wall1)
+
+    ms_t = torch.tensor([ms, kern_ms], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
+    ms, kern_ms = float(ms_t[0]), float(ms_t[1])
+    total_units = det_samples * world * args.steps
+    value = total_units / (ms / 1e3)
+
+    # ---- end to end through the public API, host (pinned) buffers, copies in the timed region
+    e2e = None
+    if not args.no_e2e:
+        e2e = run_e2e(args, w, dw, world, stream)
+
+    # ---- roofline of the dominant kernel (the fused kernel)
+    clk = clocks.get("sm_max_mhz") or 1965.0
+    peak_tflops = SMS * DFMA_PER_SM_PER_CLK * 2 * clk * 1e6 / 1e12
+    ach_tflops = F_ALG * det_samples / (kern_ms / 1e3) / 1e12
+    b_alg = algorithmic_bytes(w, det_samples)
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except (OSError, ValueError):
+        pass
+    hbm_peak = float(peaks.get("hbm_gbs", 6650.0))
+    roofline = {"bound": "alu", "achieved": ach_tflops, "peak": peak_tflops, "unit": "TFLOP/s",
+                "frac": ach_tflops / peak_tflops, "traffic": None,
+                "kernel": "pointing_to_map_kernel (fused A1-A4)", "kernel_ms": kern_ms,
+                "f_alg_per_det_sample": F_ALG,
+                "peak_note": f"fp64 pipe: {SMS} SM x {DFMA_PER_SM_PER_CLK} DFMA/clk x 2 x {clk:.0f} MHz (derived, "
+                             "B200_PROFILING.md unit counts + nvidia-smi max clock)",
+                "hbm": {"achieved_gbs": b_alg / (kern_ms / 1e3) / 1e9, "peak_gbs": hbm_peak,
+                        "frac": b_alg / (kern_ms / 1e3) / 1e9 / hbm_peak, "alg_bytes_per_launch": b_alg,
+                        "peak_note": "MEASURED_PEAKS.json hbm_gbs (measured)" if "hbm_gbs" in peaks
+                        else "fallback 6650 GB/s"}}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(args.workload)
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "config": {"workload": f"{args.workload}: {WORKLOAD_DESC[args.workload]}",
+                           "det_samples_per_rank_per_step": det_samples, "n_det": w.n_det, "n_samp": w.n_samp,
+                           "n_intervals": len(w.intervals), "nside": w.nside, "nest": w.nest, "nnz": w.nnz,
+                           "l2": f"inputs larger than L2 (TOD {w.det_data.nbytes / 1e6:.0f} MB per rank), no flush",
+                           "parallelism": f"dp{world} (one observation per rank + NCCL all-reduce of the map)"
+                           if world > 1 else "single GPU",
+                           "step": "zero map + toast_pointing_to_map" + (" + all_reduce(map)" if world > 1 else "")},
+                "clocks": clocks, "gpu_launches": args.steps, "roofline": roofline}
+        if e2e is not None:
+            line["e2e"] = e2e
+        if cpu is not None:
+            line["cpu_baseline"] = cpu
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def run_e2e(args, w, dw, world, stream):
+    """Same metric through the public binding with host buffers: H2D of the step's inputs from
+    pinned memory, the fused call, D2H of the map — all inside the timed region."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_demeurekktbb23_b200 import binding
+    pairs = []
+    for name in ("fp_quats", "boresight", "hwp", "epsilon", "det_scale", "det_data", "det_flags", "shared_flags"):
+        dev = getattr(dw, name)
+        if dev is not None:
+            pairs.append((dev.cpu().pin_memory(), dev))
+    h2d = sum(h.numel() * h.element_size() for h, _ in pairs)
+    host_map = torch.empty(dw.zmap.shape, dtype=torch.float64).pin_memory()
+    d2h = host_map.numel() * 8
+    steps = min(args.steps, 20)
+
+    def e2e_step():
+        for h, d in pairs:
+            d.copy_(h, non_blocking=True)
+        dw.zmap.zero_()
+        dw.hit_submaps.zero_()
+        dw.pointing_to_map(stream=stream)
+        if world > 1:
+            dist.all_reduce(dw.zmap, op=dist.ReduceOp.SUM)
+        host_map.copy_(dw.zmap, non_blocking=True)
+
+    for _ in range(2):
+        e2e_step()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    if world > 1:
+        dist.barrier()
+    a.record(stream)
+    for _ in range(steps):
+        e2e_step()
+    b.record(stream)
+    torch.cuda.synchronize()
+    ms = torch.tensor([a.elapsed_time(b)], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(ms, op=dist.ReduceOp.MAX)
+    ms = float(ms[0])
+    return {"value": w.det_samples * world * steps / (ms / 1e3), "unit": UNIT, "h2d_bytes_per_step": h2d,
+            "d2h_bytes_per_step": d2h, "steps": steps,
+            "path": "binding.pointing_to_map (ctypes -> toast_pointing_to_map) with pinned host inputs"}
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,371 @@
+// api.cu — the extern "C" boundary declared in include/toast_b200.h.
+//
+// Host side only: argument validation (before anything is launched), the per-device cache
+// of encoded interval work lists, and dispatch to the kernel launchers.  No exception
+// crosses the ABI; errors are returned as toast_status_t with a thread-local message.
+#include <cuda_runtime.h>
+
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/toast_b200.h"
+#include "internal.h"
+
+namespace toastb200 {
+
+namespace {
+
+thread_local std::string g_last_error;
+
+int fail(int code, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof(buf), fmt, ap);
+    va_end(ap);
+    g_last_error = buf;
+    return code;
+}
+
+int ok() {
+    g_last_error.clear();
+    return TOAST_OK;
+}
+
+int cuda_fail(cudaError_t e, const char* where) {
+    return fail(TOAST_ECUDA, "%s: %s", where, cudaGetErrorString(e));
+}
+
+// ---------------------------------------------------------------- interval work-list cache
+
+struct CacheEntry {
+    int device;
+    std::vector<toast_interval_t> intervals;
+    Chunk* d_chunks;
+    int64_t n_chunks;
+    int64_t n_samples;
+};
+
+std::mutex g_cache_mu;
+std::vector<CacheEntry> g_cache;
+constexpr size_t kCacheMax = 64;
+
+int validate_intervals(const toast_interval_t* iv, int64_t n, int64_t n_samp) {
+    if (n < 0) return fail(TOAST_EINVAL, "n_intervals < 0");
+    if (n > 0 && !iv) return fail(TOAST_EINVAL, "intervals is NULL with n_intervals > 0");
+    for (int64_t i = 0; i < n; ++i) {
+        if (iv[i].first < 0 || iv[i].last >= n_samp || iv[i].last < iv[i].first - 1)
+            return fail(TOAST_EINVAL, "interval %lld = [%lld, %lld] outside [0, n_samp=%lld)", (long long)i,
+                        (long long)iv[i].first, (long long)iv[i].last, (long long)n_samp);
+        if (i > 0 && iv[i].first <= iv[i - 1].last)
+            return fail(TOAST_EINVAL, "intervals %lld and %lld overlap or are unsorted", (long long)(i - 1),
+                        (long long)i);
+    }
+    return TOAST_OK;
+}
+
+// Returns the device work list for these intervals (creating it on first use).
+int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, WorkList* out) {
+    int rc = validate_intervals(iv, n, n_samp);
+    if (rc != TOAST_OK) return rc;
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    for (auto& c : g_cache) {
+        if (c.device == dev && (int64_t)c.intervals.size() == n &&
+            (n == 0 || std::memcmp(c.intervals.data(), iv, sizeof(toast_interval_t) * n) == 0)) {
+            *out = WorkList{c.d_chunks, c.n_chunks, c.n_samples};
+            return TOAST_OK;
+        }
+    }
+    std::vector<Chunk> chunks;
+    int64_t total = 0;
+    for (int64_t i = 0; i < n; ++i) {
+        for (int64_t f = iv[i].first; f <= iv[i].last; f += kChunk) {
+            const int64_t cnt = std::min<int64_t>(kChunk, iv[i].last - f + 1);
+            chunks.push_back(Chunk{f, (int32_t)cnt, (int32_t)i});
+            total += cnt;
+        }
+    }
+    Chunk* d = nullptr;
+    if (!chunks.empty()) {
+        e = cudaMalloc(&d, sizeof(Chunk) * chunks.size());
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(TOAST_ENOMEM, "cudaMalloc of the interval work list: %s", cudaGetErrorString(e));
+        }
+        e = cudaMemcpy(d, chunks.data(), sizeof(Chunk) * chunks.size(), cudaMemcpyHostToDevice);
+        if (e != cudaSuccess) {
+            cudaFree(d);
+            return cuda_fail(e, "cudaMemcpy of the interval work list");
+        }
+    }
+    if (g_cache.size() >= kCacheMax) {
+        int cur = dev;
+        cudaSetDevice(g_cache.front().device);
+        cudaFree(g_cache.front().d_chunks);
+        cudaSetDevice(cur);
+        g_cache.erase(g_cache.begin());
+    }
+    g_cache.push_back(CacheEntry{dev, std::vector<toast_interval_t>(iv, iv + n), d, (int64_t)chunks.size(), total});
+    *out = WorkList{d, (int64_t)chunks.size(), total};
+    return TOAST_OK;
+}
+
+bool is_pow2(int64_t x) { return x > 0 && (x & (x - 1)) == 0; }
+
+int check_nside(int64_t nside) {
+    if (!is_pow2(nside) || nside > (int64_t(1) << 29))
+        return fail(TOAST_EINVAL, "nside = %lld is not a power of two in [1, 2^29]", (long long)nside);
+    return TOAST_OK;
+}
+
+int check_submap(int64_t n_pix_submap, int64_t npix) {
+    if (n_pix_submap <= 0) return fail(TOAST_EINVAL, "n_pix_submap = %lld <= 0", (long long)n_pix_submap);
+    if (npix > 0 && npix % n_pix_submap != 0)
+        return fail(TOAST_EINVAL, "n_pix_submap = %lld does not divide npix = %lld", (long long)n_pix_submap,
+                    (long long)npix);
+    return TOAST_OK;
+}
+
+MapGeom make_map_geom(const int64_t* g2l, int64_t nps) {
+    MapGeom m;
+    m.global2local = g2l;
+    m.n_pix_submap = nps;
+    m.sm_shift = -1;
+    if (is_pow2(nps)) {
+        int sh = 0;
+        while ((int64_t(1) << sh) < nps) ++sh;
+        m.sm_shift = sh;
+    }
+    return m;
+}
+
+#define REQUIRE(ptr)                                                                 \
+    do {                                                                             \
+        if (!(ptr)) return fail(TOAST_EINVAL, "%s: required pointer " #ptr " is NULL", __func__); \
+    } while (0)
+
+#define REQUIRE_DIMS(n_det, n_samp)                                                                    \
+    do {                                                                                               \
+        if ((n_det) < 0 || (n_samp) < 0)                                                               \
+            return fail(TOAST_EINVAL, "%s: n_det = %lld, n_samp = %lld must be >= 0", __func__,        \
+                        (long long)(n_det), (long long)(n_samp));                                      \
+    } while (0)
+
+}  // namespace
+
+int num_sms() {
+    static int sms[64] = {0};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) return 148;
+    if (sms[dev] == 0) {
+        int v = 0;
+        if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || v <= 0) v = 148;
+        sms[dev] = v;
+    }
+    return sms[dev];
+}
+
+}  // namespace toastb200
+
+using namespace toastb200;
+
+extern "C" {
+
+const char* toast_last_error(void) { return g_last_error.c_str(); }
+
+const char* toast_version(void) { return "toastb200 0.1.0 (sm_100a)"; }
+
+int toast_release(void) {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    int cur = 0;
+    cudaGetDevice(&cur);
+    for (auto& c : g_cache) {
+        cudaSetDevice(c.device);
+        if (c.d_chunks) cudaFree(c.d_chunks);
+    }
+    cudaSetDevice(cur);
+    g_cache.clear();
+    return ok();
+}
+
+int toast_pointing_detector(const double* fp_quats, const double* boresight, const int32_t* quat_index,
+                            double* quats, const toast_interval_t* intervals, int64_t n_intervals,
+                            const uint8_t* shared_flags, uint8_t shared_flag_mask, int64_t n_det, int64_t n_samp,
+                            void* stream) {
+    REQUIRE_DIMS(n_det, n_samp);
+    if (n_det > 0 && n_intervals > 0) {
+        REQUIRE(fp_quats);
+        REQUIRE(boresight);
+        REQUIRE(quats);
+    }
+    WorkList wl;
+    int rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    if (rc != TOAST_OK) return rc;
+    cudaError_t e = launch_pointing_detector(wl, fp_quats, boresight, quat_index, quats, shared_flags,
+                                             shared_flag_mask, n_det, n_samp, (cudaStream_t)stream);
+    if (e != cudaSuccess) return cuda_fail(e, "pointing_detector launch");
+    return ok();
+}
+
+int toast_pixels_healpix(const int32_t* quat_index, const double* quats, const uint8_t* shared_flags,
+                         uint8_t shared_flag_mask, const int32_t* pixel_index, int64_t* pixels,
+                         const toast_interval_t* intervals, int64_t n_intervals, uint8_t* hit_submaps,
+                         int64_t n_pix_submap, int64_t nside, int nest, int64_t n_det, int64_t n_samp,
+                         void* stream) {
+    REQUIRE_DIMS(n_det, n_samp);
+    int rc = check_nside(nside);
+    if (rc != TOAST_OK) return rc;
+    if (nest != 0 && nest != 1) return fail(TOAST_EINVAL, "nest = %d must be 0 (RING) or 1 (NESTED)", nest);
+    rc = check_submap(n_pix_submap, 12 * nside * nside);
+    if (rc != TOAST_OK) return rc;
+    if (n_det > 0 && n_intervals > 0) {
+        REQUIRE(quats);
+        REQUIRE(pixels);
+    }
+    WorkList wl;
+    rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    if (rc != TOAST_OK) return rc;
+    cudaError_t e = launch_pixels_healpix(wl, quat_index, quats, shared_flags, shared_flag_mask, pixel_index, pixels,
+                                          hit_submaps, n_pix_submap, nside, nest, n_det, n_samp,
+                                          (cudaStream_t)stream);
+    if (e != cudaSuccess) return cuda_fail(e, "pixels_healpix launch");
+    return ok();
+}
+
+int toast_stokes_weights_iqu(const int32_t* quat_index, const double* quats, const int32_t* weight_index,
+                             double* weights, const double* hwp, const double* epsilon, double cal,
+                             const toast_interval_t* intervals, int64_t n_intervals, int64_t n_det, int64_t n_samp,
+                             void* stream) {
+    REQUIRE_DIMS(n_det, n_samp);
+    if (n_det > 0 && n_intervals > 0) {
+        REQUIRE(quats);
+        REQUIRE(weights);
+        REQUIRE(epsilon);
+    }
+    WorkList wl;
+    int rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    if (rc != TOAST_OK) return rc;
+    cudaError_t e = launch_stokes_weights_iqu(wl, quat_index, quats, weight_index, weights, hwp, epsilon, cal, n_det,
+                                              n_samp, (cudaStream_t)stream);
+    if (e != cudaSuccess) return cuda_fail(e, "stokes_weights_iqu launch");
+    return ok();
+}
+
+int toast_build_noise_weighted(const int64_t* global2local, double* zmap, int64_t n_pix_submap, int64_t nnz,
+                               const int32_t* pixel_index, const int64_t* pixels, const int32_t* weight_index,
+                               const double* weights, const int32_t* data_index, const double* det_data,
+                               const int32_t* flag_index, const uint8_t* det_flags, uint8_t det_flag_mask,
+                               const double* det_scale, const uint8_t* shared_flags, uint8_t shared_flag_mask,
+                               const toast_interval_t* intervals, int64_t n_intervals, int64_t n_det, int64_t n_samp,
+                               void* stream) {
+    REQUIRE_DIMS(n_det, n_samp);
+    if (nnz != 1 && nnz != 3) return fail(TOAST_EINVAL, "nnz = %lld must be 1 or 3", (long long)nnz);
+    int rc = check_submap(n_pix_submap, 0);
+    if (rc != TOAST_OK) return rc;
+    if (n_det > 0 && n_intervals > 0) {
+        REQUIRE(global2local);
+        REQUIRE(zmap);
+        REQUIRE(pixels);
+        REQUIRE(weights);
+        REQUIRE(det_data);
+        REQUIRE(det_scale);
+    }
+    WorkList wl;
+    rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    if (rc != TOAST_OK) return rc;
+    cudaError_t e = launch_build_noise_weighted(wl, make_map_geom(global2local, n_pix_submap), zmap, (int)nnz,
+                                                pixel_index, pixels, weight_index, weights, data_index, det_data,
+                                                flag_index, det_flags, det_flag_mask, det_scale, shared_flags,
+                                                shared_flag_mask, n_det, n_samp, (cudaStream_t)stream);
+    if (e != cudaSuccess) return cuda_fail(e, "build_noise_weighted launch");
+    return ok();
+}
+
+int toast_scan_map(const int64_t* global2local, int64_t n_pix_submap, const double* mapdata, int64_t nnz,
+                   const int32_t* data_index, double* det_data, const int32_t* pixel_index, const int64_t* pixels,
+                   const int32_t* weight_index, const double* weights, const toast_interval_t* intervals,
+                   int64_t n_intervals, double data_scale, int should_zero, int should_subtract, int64_t n_det,
+                   int64_t n_samp, void* stream) {
+    REQUIRE_DIMS(n_det, n_samp);
+    if (nnz != 1 && nnz != 3) return fail(TOAST_EINVAL, "nnz = %lld must be 1 or 3", (long long)nnz);
+    int rc = check_submap(n_pix_submap, 0);
+    if (rc != TOAST_OK) return rc;
+    if (n_det > 0 && n_intervals > 0) {
+        REQUIRE(global2local);
+        REQUIRE(mapdata);
+        REQUIRE(det_data);
+        REQUIRE(pixels);
+        REQUIRE(weights);
+    }
+    WorkList wl;
+    rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    if (rc != TOAST_OK) return rc;
+    cudaError_t e = launch_scan_map(wl, make_map_geom(global2local, n_pix_submap), mapdata, (int)nnz, data_index,
+                                    det_data, pixel_index, pixels, weight_index, weights, data_scale, should_zero,
+                                    should_subtract, n_det, n_samp, (cudaStream_t)stream);
+    if (e != cudaSuccess) return cuda_fail(e, "scan_map launch");
+    return ok();
+}
+
+int toast_pointing_to_map(const double* fp_quats, const double* boresight, const double* hwp, const double* epsilon,
+                          double cal, const double* det_scale, const double* det_data, const uint8_t* det_flags,
+                          uint8_t det_flag_mask, const uint8_t* shared_flags, uint8_t shared_flag_mask,
+                          const toast_interval_t* intervals, int64_t n_intervals, int64_t nside, int nest,
+                          int64_t nnz, const int64_t* global2local, int64_t n_pix_submap, double* zmap,
+                          uint8_t* hit_submaps, int64_t* pixels_out, double* weights_out, int64_t n_det,
+                          int64_t n_samp, void* stream) {
+    REQUIRE_DIMS(n_det, n_samp);
+    int rc = check_nside(nside);
+    if (rc != TOAST_OK) return rc;
+    if (nest != 0 && nest != 1) return fail(TOAST_EINVAL, "nest = %d must be 0 (RING) or 1 (NESTED)", nest);
+    if (nnz != 1 && nnz != 3) return fail(TOAST_EINVAL, "nnz = %lld must be 1 or 3", (long long)nnz);
+    rc = check_submap(n_pix_submap, 12 * nside * nside);
+    if (rc != TOAST_OK) return rc;
+    if (n_det > 0 && n_intervals > 0) {
+        REQUIRE(fp_quats);
+        REQUIRE(boresight);
+        REQUIRE(epsilon);
+        REQUIRE(det_scale);
+        REQUIRE(det_data);
+        REQUIRE(global2local);
+        REQUIRE(zmap);
+    }
+    WorkList wl;
+    rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    if (rc != TOAST_OK) return rc;
+    FusedArgs a;
+    a.fp_quats = fp_quats;
+    a.boresight = boresight;
+    a.hwp = hwp;
+    a.epsilon = epsilon;
+    a.cal = cal;
+    a.det_scale = det_scale;
+    a.det_data = det_data;
+    a.det_flags = det_flags;
+    a.det_flag_mask = det_flag_mask;
+    a.shared_flags = shared_flags;
+    a.shared_flag_mask = shared_flag_mask;
+    a.nside = nside;
+    a.nest = nest;
+    a.nnz = (int)nnz;
+    a.map = make_map_geom(global2local, n_pix_submap);
+    a.zmap = zmap;
+    a.hit_submaps = hit_submaps;
+    a.pixels_out = pixels_out;
+    a.weights_out = weights_out;
+    a.n_det = n_det;
+    a.n_samp = n_samp;
+    cudaError_t e = launch_pointing_to_map(wl, a, (cudaStream_t)stream);
+    if (e != cudaSuccess) return cuda_fail(e, "pointing_to_map launch");
+    return ok();
+}
+
+}  // extern "C"

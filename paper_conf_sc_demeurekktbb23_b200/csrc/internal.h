@@ -1,0 +1,87 @@
+// internal.h — launch-side types shared by api.cu and the kernel files (not part of the ABI).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "../../include/toast_b200.h"
+
+namespace toastb200 {
+
+// Samples per work chunk = threads per CTA of every kernel (one sample per thread).
+constexpr int kChunk = 256;
+// Detectors per fused work item (a CTA loops over them with the sample's boresight
+// rotation held in registers).
+constexpr int kDetBlock = 32;
+
+// One chunk of <= kChunk consecutive in-interval samples (never crosses an interval).
+struct Chunk {
+    int64_t first;
+    int32_t count;
+    int32_t interval;
+};
+
+struct WorkList {
+    const Chunk* chunks;  // device
+    int64_t n_chunks;
+    int64_t n_samples;    // total in-interval samples
+};
+
+struct MapGeom {
+    const int64_t* global2local;
+    int64_t n_pix_submap;
+    int sm_shift;         // log2(n_pix_submap) if a power of two, else -1
+};
+
+struct FusedArgs {
+    const double* fp_quats;
+    const double* boresight;
+    const double* hwp;
+    const double* epsilon;
+    double cal;
+    const double* det_scale;
+    const double* det_data;
+    const uint8_t* det_flags;
+    uint8_t det_flag_mask;
+    const uint8_t* shared_flags;
+    uint8_t shared_flag_mask;
+    int64_t nside;
+    int nest;
+    int nnz;
+    MapGeom map;
+    double* zmap;
+    uint8_t* hit_submaps;
+    int64_t* pixels_out;
+    double* weights_out;
+    int64_t n_det;
+    int64_t n_samp;
+};
+
+cudaError_t launch_pointing_detector(const WorkList& wl, const double* fp_quats, const double* boresight,
+                                     const int32_t* quat_index, double* quats, const uint8_t* shared_flags,
+                                     uint8_t shared_flag_mask, int64_t n_det, int64_t n_samp, cudaStream_t st);
+cudaError_t launch_pixels_healpix(const WorkList& wl, const int32_t* quat_index, const double* quats,
+                                  const uint8_t* shared_flags, uint8_t shared_flag_mask, const int32_t* pixel_index,
+                                  int64_t* pixels, uint8_t* hit_submaps, int64_t n_pix_submap, int64_t nside,
+                                  int nest, int64_t n_det, int64_t n_samp, cudaStream_t st);
+cudaError_t launch_stokes_weights_iqu(const WorkList& wl, const int32_t* quat_index, const double* quats,
+                                      const int32_t* weight_index, double* weights, const double* hwp,
+                                      const double* epsilon, double cal, int64_t n_det, int64_t n_samp,
+                                      cudaStream_t st);
+cudaError_t launch_build_noise_weighted(const WorkList& wl, const MapGeom& mg, double* zmap, int nnz,
+                                        const int32_t* pixel_index, const int64_t* pixels,
+                                        const int32_t* weight_index, const double* weights,
+                                        const int32_t* data_index, const double* det_data,
+                                        const int32_t* flag_index, const uint8_t* det_flags, uint8_t det_flag_mask,
+                                        const double* det_scale, const uint8_t* shared_flags,
+                                        uint8_t shared_flag_mask, int64_t n_det, int64_t n_samp, cudaStream_t st);
+cudaError_t launch_scan_map(const WorkList& wl, const MapGeom& mg, const double* mapdata, int nnz,
+                            const int32_t* data_index, double* det_data, const int32_t* pixel_index,
+                            const int64_t* pixels, const int32_t* weight_index, const double* weights,
+                            double data_scale, int should_zero, int should_subtract, int64_t n_det, int64_t n_samp,
+                            cudaStream_t st);
+cudaError_t launch_pointing_to_map(const WorkList& wl, const FusedArgs& a, cudaStream_t st);
+
+int num_sms();
+
+}  // namespace toastb200

@@ -1,0 +1,296 @@
+// unfused.cu — the five TOAST kernels as separate sm_100a launches (A1-A5).
+//
+// Iteration space: detector x interval x sample.  The host encodes the
+// intervals into a list of <= 256-sample chunks; a CTA is (chunk, detector) and a thread is
+// one sample, so every HBM stream (boresight, quaternions, pixels, weights, TOD) is read
+// and written coalesced along the sample axis; out-of-interval samples are never touched
+// (PAPER.md:143).  These kernels are HBM-bound.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+
+#include "device_math.cuh"
+#include "internal.h"
+#include "map_accum.cuh"
+
+namespace toastb200 {
+
+namespace {
+
+__device__ __forceinline__ void load_quat(const double* __restrict__ p, double q[4]) {
+    const double2 lo = __ldg(reinterpret_cast<const double2*>(p));
+    const double2 hi = __ldg(reinterpret_cast<const double2*>(p) + 1);
+    q[0] = lo.x; q[1] = lo.y; q[2] = hi.x; q[3] = hi.y;
+}
+
+__device__ __forceinline__ int64_t row_of(const int32_t* __restrict__ index, int64_t d) {
+    return index ? (int64_t)__ldg(&index[d]) : d;
+}
+
+dim3 grid_for(const WorkList& wl, int64_t n_det) {
+    const unsigned gx = (unsigned)std::min<int64_t>(wl.n_chunks, 0x7fffffff);
+    const unsigned gy = (unsigned)std::min<int64_t>(n_det, 65535);
+    return dim3(gx, gy, 1);
+}
+
+// ----------------------------------------------------------------------------- A1
+
+__global__ void __launch_bounds__(kChunk) pointing_detector_kernel(
+    const Chunk* __restrict__ chunks, int64_t n_chunks, const double* __restrict__ fp_quats,
+    const double* __restrict__ boresight, const int32_t* __restrict__ quat_index, double* __restrict__ quats,
+    const uint8_t* __restrict__ shared_flags, uint8_t shared_flag_mask, int64_t n_det, int64_t n_samp) {
+    for (int64_t c = blockIdx.x; c < n_chunks; c += gridDim.x) {
+        const Chunk ch = chunks[c];
+        if ((int)threadIdx.x >= ch.count) continue;
+        const int64_t s = ch.first + threadIdx.x;
+        double b[4];
+        if (shared_flags && (__ldg(&shared_flags[s]) & shared_flag_mask)) {
+            b[0] = 0.0; b[1] = 0.0; b[2] = 0.0; b[3] = 1.0;  // reading S2
+        } else {
+            load_quat(boresight + 4 * s, b);
+        }
+        for (int64_t d = blockIdx.y; d < n_det; d += gridDim.y) {
+            double f[4], q[4];
+            load_quat(fp_quats + 4 * d, f);
+            quat_mul(b, f, q);
+            double2* out = reinterpret_cast<double2*>(quats + (row_of(quat_index, d) * n_samp + s) * 4);
+            out[0] = make_double2(q[0], q[1]);
+            out[1] = make_double2(q[2], q[3]);
+        }
+    }
+}
+
+// ----------------------------------------------------------------------------- A2
+
+template <bool NEST>
+__global__ void __launch_bounds__(kChunk) pixels_healpix_kernel(
+    const Chunk* __restrict__ chunks, int64_t n_chunks, const int32_t* __restrict__ quat_index,
+    const double* __restrict__ quats, const uint8_t* __restrict__ shared_flags, uint8_t shared_flag_mask,
+    const int32_t* __restrict__ pixel_index, int64_t* __restrict__ pixels, uint8_t* __restrict__ hit_submaps,
+    int64_t n_pix_submap, HealpixGeom g, int64_t n_det, int64_t n_samp) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t c = blockIdx.x; c < n_chunks; c += gridDim.x) {
+        const Chunk ch = chunks[c];
+        if ((int)(threadIdx.x & ~31u) >= ch.count) continue;  // whole warp out of range
+        const bool in = (int)threadIdx.x < ch.count;
+        const int64_t s = ch.first + threadIdx.x;
+        const bool flagged = in && shared_flags && (__ldg(&shared_flags[s]) & shared_flag_mask);
+        for (int64_t d = blockIdx.y; d < n_det; d += gridDim.y) {
+            int64_t pix = -1;
+            if (in && !flagged) {
+                double q[4];
+                load_quat(quats + (row_of(quat_index, d) * n_samp + s) * 4, q);
+                // dir = R(q) z = third column of R(q)
+                const double dx = 2.0 * (q[0] * q[2] + q[1] * q[3]);
+                const double dy = 2.0 * (q[1] * q[2] - q[0] * q[3]);
+                const double dz = 1.0 - 2.0 * (q[0] * q[0] + q[1] * q[1]);
+                pix = vec2pix<NEST>(g, dx, dy, dz);
+            }
+            if (in) pixels[row_of(pixel_index, d) * n_samp + s] = pix;
+            if (hit_submaps) {
+                const int64_t sm = pix >= 0 ? pix / n_pix_submap : -1;
+                const int64_t prev = __shfl_up_sync(kFull, sm, 1);
+                if (sm >= 0 && (lane == 0 || prev != sm)) hit_submaps[sm] = 1;
+            }
+        }
+    }
+}
+
+// ----------------------------------------------------------------------------- A3
+
+template <bool HWP>
+__global__ void __launch_bounds__(kChunk) stokes_weights_kernel(
+    const Chunk* __restrict__ chunks, int64_t n_chunks, const int32_t* __restrict__ quat_index,
+    const double* __restrict__ quats, const int32_t* __restrict__ weight_index, double* __restrict__ weights,
+    const double* __restrict__ hwp, const double* __restrict__ epsilon, double cal, int64_t n_det, int64_t n_samp) {
+    for (int64_t c = blockIdx.x; c < n_chunks; c += gridDim.x) {
+        const Chunk ch = chunks[c];
+        if ((int)threadIdx.x >= ch.count) continue;
+        const int64_t s = ch.first + threadIdx.x;
+        double c4 = 1.0, s4 = 0.0;
+        if (HWP) sincos(4.0 * __ldg(&hwp[s]), &s4, &c4);
+        for (int64_t d = blockIdx.y; d < n_det; d += gridDim.y) {
+            double q[4];
+            load_quat(quats + (row_of(quat_index, d) * n_samp + s) * 4, q);
+            // bx = (R x)_z, by = -(R y)_z: third row of R(q) (orthonormal detector frame)
+            const double bx = 2.0 * (q[0] * q[2] - q[1] * q[3]);
+            const double by = -2.0 * (q[1] * q[2] + q[0] * q[3]);
+            double c2, s2;
+            cos_sin_2psi(bx, by, c2, s2);
+            const double eps = __ldg(&epsilon[d]);
+            const double etacal = (1.0 - eps) / (1.0 + eps) * cal;
+            double cq = c2, sq = s2;
+            if (HWP) {
+                cq = c2 * c4 - s2 * s4;
+                sq = s2 * c4 + c2 * s4;
+            }
+            double* out = weights + (row_of(weight_index, d) * n_samp + s) * 3;
+            out[0] = cal;
+            out[1] = etacal * cq;
+            out[2] = etacal * sq;
+        }
+    }
+}
+
+// ----------------------------------------------------------------------------- A4
+
+template <int NNZ>
+__global__ void __launch_bounds__(kChunk) build_noise_weighted_kernel(
+    const Chunk* __restrict__ chunks, int64_t n_chunks, MapGeom mg, double* __restrict__ zmap,
+    const int32_t* __restrict__ pixel_index, const int64_t* __restrict__ pixels,
+    const int32_t* __restrict__ weight_index, const double* __restrict__ weights,
+    const int32_t* __restrict__ data_index, const double* __restrict__ det_data,
+    const int32_t* __restrict__ flag_index, const uint8_t* __restrict__ det_flags, uint8_t det_flag_mask,
+    const double* __restrict__ det_scale, const uint8_t* __restrict__ shared_flags, uint8_t shared_flag_mask,
+    int64_t n_det, int64_t n_samp) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t c = blockIdx.x; c < n_chunks; c += gridDim.x) {
+        const Chunk ch = chunks[c];
+        if ((int)(threadIdx.x & ~31u) >= ch.count) continue;
+        const bool in = (int)threadIdx.x < ch.count;
+        const int64_t s = ch.first + threadIdx.x;
+        const bool sflag = in && shared_flags && (__ldg(&shared_flags[s]) & shared_flag_mask);
+        for (int64_t d = blockIdx.y; d < n_det; d += gridDim.y) {
+            int64_t key = -1 - lane;
+            double v0 = 0.0, v1 = 0.0, v2 = 0.0;
+            if (in && !sflag) {
+                const int64_t pix = __ldg(&pixels[row_of(pixel_index, d) * n_samp + s]);
+                const bool dflag = det_flags && (__ldg(&det_flags[row_of(flag_index, d) * n_samp + s]) & det_flag_mask);
+                if (pix >= 0 && !dflag) {
+                    key = pix;
+                    const double scaled = __ldg(&det_scale[d]) * __ldg(&det_data[row_of(data_index, d) * n_samp + s]);
+                    const double* w = weights + (row_of(weight_index, d) * n_samp + s) * NNZ;
+                    v0 = scaled * __ldg(&w[0]);
+                    if (NNZ == 3) {
+                        v1 = scaled * __ldg(&w[1]);
+                        v2 = scaled * __ldg(&w[2]);
+                    }
+                }
+            }
+            warp_accumulate<NNZ>(key, v0, v1, v2, mg, zmap, nullptr);
+        }
+    }
+}
+
+// ----------------------------------------------------------------------------- A5
+
+template <int NNZ>
+__global__ void __launch_bounds__(kChunk) scan_map_kernel(
+    const Chunk* __restrict__ chunks, int64_t n_chunks, MapGeom mg, const double* __restrict__ mapdata,
+    const int32_t* __restrict__ data_index, double* __restrict__ det_data, const int32_t* __restrict__ pixel_index,
+    const int64_t* __restrict__ pixels, const int32_t* __restrict__ weight_index, const double* __restrict__ weights,
+    double data_scale, int should_zero, int should_subtract, int64_t n_det, int64_t n_samp) {
+    for (int64_t c = blockIdx.x; c < n_chunks; c += gridDim.x) {
+        const Chunk ch = chunks[c];
+        if ((int)threadIdx.x >= ch.count) continue;
+        const int64_t s = ch.first + threadIdx.x;
+        for (int64_t d = blockIdx.y; d < n_det; d += gridDim.y) {
+            const int64_t pix = __ldg(&pixels[row_of(pixel_index, d) * n_samp + s]);
+            if (pix < 0) continue;
+            int64_t sm, lp;
+            if (mg.sm_shift >= 0) {
+                sm = pix >> mg.sm_shift;
+                lp = pix & (mg.n_pix_submap - 1);
+            } else {
+                sm = pix / mg.n_pix_submap;
+                lp = pix - sm * mg.n_pix_submap;
+            }
+            const int64_t loc = __ldg(&mg.global2local[sm]);
+            if (loc < 0) continue;
+            const double* m = mapdata + (loc * mg.n_pix_submap + lp) * NNZ;
+            const double* w = weights + (row_of(weight_index, d) * n_samp + s) * NNZ;
+            double t = __ldg(&m[0]) * __ldg(&w[0]);
+            if (NNZ == 3) {
+                t += __ldg(&m[1]) * __ldg(&w[1]);
+                t += __ldg(&m[2]) * __ldg(&w[2]);
+            }
+            t *= data_scale;
+            double* tod = det_data + row_of(data_index, d) * n_samp + s;
+            const double base = should_zero ? 0.0 : *tod;
+            *tod = should_subtract ? base - t : base + t;
+        }
+    }
+}
+
+}  // namespace
+
+cudaError_t launch_pointing_detector(const WorkList& wl, const double* fp_quats, const double* boresight,
+                                     const int32_t* quat_index, double* quats, const uint8_t* shared_flags,
+                                     uint8_t shared_flag_mask, int64_t n_det, int64_t n_samp, cudaStream_t st) {
+    if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
+    pointing_detector_kernel<<<grid_for(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, fp_quats, boresight,
+                                                                      quat_index, quats, shared_flags,
+                                                                      shared_flag_mask, n_det, n_samp);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_pixels_healpix(const WorkList& wl, const int32_t* quat_index, const double* quats,
+                                  const uint8_t* shared_flags, uint8_t shared_flag_mask, const int32_t* pixel_index,
+                                  int64_t* pixels, uint8_t* hit_submaps, int64_t n_pix_submap, int64_t nside,
+                                  int nest, int64_t n_det, int64_t n_samp, cudaStream_t st) {
+    if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
+    const HealpixGeom g = make_geom(nside);
+    if (nest)
+        pixels_healpix_kernel<true><<<grid_for(wl, n_det), kChunk, 0, st>>>(
+            wl.chunks, wl.n_chunks, quat_index, quats, shared_flags, shared_flag_mask, pixel_index, pixels,
+            hit_submaps, n_pix_submap, g, n_det, n_samp);
+    else
+        pixels_healpix_kernel<false><<<grid_for(wl, n_det), kChunk, 0, st>>>(
+            wl.chunks, wl.n_chunks, quat_index, quats, shared_flags, shared_flag_mask, pixel_index, pixels,
+            hit_submaps, n_pix_submap, g, n_det, n_samp);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_stokes_weights_iqu(const WorkList& wl, const int32_t* quat_index, const double* quats,
+                                      const int32_t* weight_index, double* weights, const double* hwp,
+                                      const double* epsilon, double cal, int64_t n_det, int64_t n_samp,
+                                      cudaStream_t st) {
+    if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
+    if (hwp)
+        stokes_weights_kernel<true><<<grid_for(wl, n_det), kChunk, 0, st>>>(
+            wl.chunks, wl.n_chunks, quat_index, quats, weight_index, weights, hwp, epsilon, cal, n_det, n_samp);
+    else
+        stokes_weights_kernel<false><<<grid_for(wl, n_det), kChunk, 0, st>>>(
+            wl.chunks, wl.n_chunks, quat_index, quats, weight_index, weights, hwp, epsilon, cal, n_det, n_samp);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_build_noise_weighted(const WorkList& wl, const MapGeom& mg, double* zmap, int nnz,
+                                        const int32_t* pixel_index, const int64_t* pixels,
+                                        const int32_t* weight_index, const double* weights,
+                                        const int32_t* data_index, const double* det_data,
+                                        const int32_t* flag_index, const uint8_t* det_flags, uint8_t det_flag_mask,
+                                        const double* det_scale, const uint8_t* shared_flags,
+                                        uint8_t shared_flag_mask, int64_t n_det, int64_t n_samp, cudaStream_t st) {
+    if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
+    if (nnz == 3)
+        build_noise_weighted_kernel<3><<<grid_for(wl, n_det), kChunk, 0, st>>>(
+            wl.chunks, wl.n_chunks, mg, zmap, pixel_index, pixels, weight_index, weights, data_index, det_data,
+            flag_index, det_flags, det_flag_mask, det_scale, shared_flags, shared_flag_mask, n_det, n_samp);
+    else
+        build_noise_weighted_kernel<1><<<grid_for(wl, n_det), kChunk, 0, st>>>(
+            wl.chunks, wl.n_chunks, mg, zmap, pixel_index, pixels, weight_index, weights, data_index, det_data,
+            flag_index, det_flags, det_flag_mask, det_scale, shared_flags, shared_flag_mask, n_det, n_samp);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_scan_map(const WorkList& wl, const MapGeom& mg, const double* mapdata, int nnz,
+                            const int32_t* data_index, double* det_data, const int32_t* pixel_index,
+                            const int64_t* pixels, const int32_t* weight_index, const double* weights,
+                            double data_scale, int should_zero, int should_subtract, int64_t n_det, int64_t n_samp,
+                            cudaStream_t st) {
+    if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
+    if (nnz == 3)
+        scan_map_kernel<3><<<grid_for(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, mg, mapdata, data_index,
+                                                                    det_data, pixel_index, pixels, weight_index,
+                                                                    weights, data_scale, should_zero,
+                                                                    should_subtract, n_det, n_samp);
+    else
+        scan_map_kernel<1><<<grid_for(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, mg, mapdata, data_index,
+                                                                    det_data, pixel_index, pixels, weight_index,
+                                                                    weights, data_scale, should_zero,
+                                                                    should_subtract, n_det, n_samp);
+    return cudaGetLastError();
+}
+
+}  // namespace toastb200
