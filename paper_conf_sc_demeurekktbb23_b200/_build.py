@@ -14,7 +14,6 @@ NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",
     "-O3", "-lineinfo", "-std=c++17",
     "-Xcompiler", "-fPIC", "-shared",
-    "-Xptxas", "-warn-spills",
 ]
 
 
@@ -51,3 +50,14 @@ def build(force: bool = False, verbose: bool = False) -> str:
 
 if __name__ == "__main__":
     print(build(force=True, verbose=True))
+
+
+def build_variant(name: str, defines: dict, out_dir: str = None) -> str:
+    """Build a tuning variant of the library with extra -D macros (not used by the product path)."""
+    out_dir = out_dir or os.path.join(os.path.dirname(HERE), "build", "variants")
+    os.makedirs(out_dir, exist_ok=True)
+    out = os.path.join(out_dir, f"libtoastb200_{name}.so")
+    nvcc = "/usr/local/cuda/bin/nvcc" if os.path.exists("/usr/local/cuda/bin/nvcc") else "nvcc"
+    cmd = [nvcc, *NVCC_FLAGS, *[f"-D{k}={v}" for k, v in defines.items()], "-o", out, *sources()]
+    subprocess.check_call(cmd)
+    return out

@@ -38,10 +38,11 @@ def load():
     global _lib
     if _lib is not None:
         return _lib
-    if not os.path.exists(_build.LIB):
-        raise ToastError(f"{_build.LIB} is missing: run `python -c 'import __graft_entry__ as g; g.build()'` "
+    path = os.environ.get("TOASTB200_LIB", _build.LIB)  # tuning experiments may point at a variant build
+    if not os.path.exists(path):
+        raise ToastError(f"{path} is missing: run `python -c 'import __graft_entry__ as g; g.build()'` "
                          "(there is no CPU fallback)")
-    L = ctypes.CDLL(_build.LIB)
+    L = ctypes.CDLL(path)
     L.toast_last_error.restype = ctypes.c_char_p
     L.toast_version.restype = ctypes.c_char_p
     L.toast_release.restype = I32

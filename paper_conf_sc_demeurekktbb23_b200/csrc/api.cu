@@ -44,6 +44,7 @@ int cuda_fail(cudaError_t e, const char* where) {
 
 struct CacheEntry {
     int device;
+    int chunk;
     std::vector<toast_interval_t> intervals;
     Chunk* d_chunks;
     int64_t n_chunks;
@@ -69,7 +70,7 @@ int validate_intervals(const toast_interval_t* iv, int64_t n, int64_t n_samp) {
 }
 
 // Returns the device work list for these intervals (creating it on first use).
-int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, WorkList* out) {
+int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, WorkList* out, int chunk = kChunk) {
     int rc = validate_intervals(iv, n, n_samp);
     if (rc != TOAST_OK) return rc;
     int dev = 0;
@@ -77,7 +78,7 @@ int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, WorkList
     if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
     std::lock_guard<std::mutex> lk(g_cache_mu);
     for (auto& c : g_cache) {
-        if (c.device == dev && (int64_t)c.intervals.size() == n &&
+        if (c.device == dev && c.chunk == chunk && (int64_t)c.intervals.size() == n &&
             (n == 0 || std::memcmp(c.intervals.data(), iv, sizeof(toast_interval_t) * n) == 0)) {
             *out = WorkList{c.d_chunks, c.n_chunks, c.n_samples};
             return TOAST_OK;
@@ -86,8 +87,8 @@ int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, WorkList
     std::vector<Chunk> chunks;
     int64_t total = 0;
     for (int64_t i = 0; i < n; ++i) {
-        for (int64_t f = iv[i].first; f <= iv[i].last; f += kChunk) {
-            const int64_t cnt = std::min<int64_t>(kChunk, iv[i].last - f + 1);
+        for (int64_t f = iv[i].first; f <= iv[i].last; f += chunk) {
+            const int64_t cnt = std::min<int64_t>(chunk, iv[i].last - f + 1);
             chunks.push_back(Chunk{f, (int32_t)cnt, (int32_t)i});
             total += cnt;
         }
@@ -112,7 +113,8 @@ int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, WorkList
         cudaSetDevice(cur);
         g_cache.erase(g_cache.begin());
     }
-    g_cache.push_back(CacheEntry{dev, std::vector<toast_interval_t>(iv, iv + n), d, (int64_t)chunks.size(), total});
+    g_cache.push_back(
+        CacheEntry{dev, chunk, std::vector<toast_interval_t>(iv, iv + n), d, (int64_t)chunks.size(), total});
     *out = WorkList{d, (int64_t)chunks.size(), total};
     return TOAST_OK;
 }
@@ -159,6 +161,31 @@ MapGeom make_map_geom(const int64_t* g2l, int64_t nps) {
     } while (0)
 
 }  // namespace
+
+// Per-device pool of work-distribution counters, handed out round robin so that launches
+// in flight on different streams use different counters.
+unsigned long long* sched_counter(int* err) {
+    constexpr int kPool = 64;
+    static std::mutex mu;
+    static unsigned long long* pools[64] = {nullptr};
+    static unsigned next[64] = {0};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) {
+        *err = 1;
+        return nullptr;
+    }
+    std::lock_guard<std::mutex> lk(mu);
+    if (!pools[dev]) {
+        if (cudaMalloc(&pools[dev], kPool * 128) != cudaSuccess) {  // one 128-B line per counter
+            cudaGetLastError();
+            *err = 1;
+            return nullptr;
+        }
+        cudaMemset(pools[dev], 0, kPool * 128);
+    }
+    *err = 0;
+    return pools[dev] + (next[dev]++ % kPool) * (128 / sizeof(unsigned long long));
+}
 
 int num_sms() {
     static int sms[64] = {0};
@@ -339,7 +366,7 @@ int toast_pointing_to_map(const double* fp_quats, const double* boresight, const
         REQUIRE(zmap);
     }
     WorkList wl;
-    rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    rc = get_worklist(intervals, n_intervals, n_samp, &wl, kFusedChunk);
     if (rc != TOAST_OK) return rc;
     FusedArgs a;
     a.fp_quats = fp_quats;
@@ -363,7 +390,10 @@ int toast_pointing_to_map(const double* fp_quats, const double* boresight, const
     a.weights_out = weights_out;
     a.n_det = n_det;
     a.n_samp = n_samp;
-    cudaError_t e = launch_pointing_to_map(wl, a, (cudaStream_t)stream);
+    int serr = 0;
+    unsigned long long* sched = sched_counter(&serr);
+    if (serr) return fail(TOAST_ENOMEM, "could not allocate the work-distribution counter");
+    cudaError_t e = launch_pointing_to_map(wl, a, sched, (cudaStream_t)stream);
     if (e != cudaSuccess) return cuda_fail(e, "pointing_to_map launch");
     return ok();
 }

@@ -22,6 +22,136 @@ namespace toastb200 {
 constexpr double kTwoThird = 2.0 / 3.0;
 constexpr double kInvHalfPi = 0.6366197723675813430755350534900574;  // 2/pi
 
+// (2/pi) atan(t) = t P(t^2) on |t| <= tan(pi/8); coefficients from scripts/fit_atan.py
+// (Chebyshev interpolant, max relative error 1.2e-16 in exact arithmetic).
+static __constant__ double kAtanQ[11] = {
+    0x1.45f306dc9c882p-1,  // 0.63661977236758127
+    -0x1.b2995e7b7b1bfp-3,  // -0.21220659078916346
+    0x1.04c26be371b2ap-3,  // 0.12732395446638495
+    -0x1.7483756164e14p-4,  // -0.090945681111684273
+    0x1.21bb8c039cd9ap-4,  // 0.070735499315381395
+    -0x1.da19e12de59d2p-5,  // -0.057873668483057764
+    0x1.910bf286e9087p-5,  // 0.048955892262967864
+    -0x1.5a4f32beaf656p-5,  // -0.042274092780172509
+    0x1.28b3704d8f8cdp-5,  // 0.036218375531903747
+    -0x1.c5c0e72211c3bp-6,  // -0.027694917407895963
+    0x1.b97329ffc867cp-7,  // 0.013471980578802382
+};
+
+constexpr double kTanPi8 = 0.41421356237309504880;
+
+// 1/x for finite x > 0 (no IEEE rounding guarantee; <= ~1 ulp): MUFU seed + 2 Newton steps.
+__device__ __forceinline__ double fast_rcp(double x) {
+    double r;
+    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(x));
+    r = fma(r, fma(-x, r, 1.0), r);
+    r = fma(r, fma(-x, r, 1.0), r);
+    return r;
+}
+
+// tt = fmodulo(2 atan2(y, x) / pi, 4) in [0, 4) -- the HEALPix longitude in quarter turns --
+// with tt = 0 at x = y = 0 (reading S3).
+// Octant reduction with ONE reciprocal: with mx = max(|x|,|y|), mn = min(|x|,|y|) and
+// beta = [mn > tan(pi/8) mx], t = (mn - beta mx) / (mx + beta mn) lies in [-tan(pi/8),
+// tan(pi/8)] and tau = (2/pi) atan(t) = t P(t^2).  The octant bookkeeping is integer: the
+// result is tt = K/2 + S tau with K in 0..8 and S = +-1, evaluated by ONE fma, so the
+// octant offsets (multiples of 1/2 quarter turn) are exact.  Absolute error ~3e-16 quarter
+// turns: it differs from a correctly rounded atan2 only at the last-ulp level, so HEALPix
+// floors can differ from the oracle's only for directions within ~1e-15 rad of a pixel
+// boundary (rule T1 allows 1e-12 rad).
+//
+// Two phases so that callers can share ONE reciprocal between the longitude and the
+// polarisation weights (the MUFU/XU pipe, not the FP64 pipe, is the scarce unit on B200).
+struct QtPrep {
+    double num, den;  // t = num / den
+    int kk;           // octant offset in half quarter turns
+    bool neg;         // sign S
+};
+
+__device__ __forceinline__ QtPrep qt_prepare(double x, double y) {
+    const double ax = fabs(x), ay = fabs(y);
+    const bool swap = ay > ax;
+    const double mx = swap ? ay : ax;
+    const double mn = swap ? ax : ay;
+    const bool big = mn > kTanPi8 * mx;
+    const double beta = big ? 1.0 : 0.0;
+    QtPrep q;
+    q.num = fma(-beta, mx, mn);
+    q.den = fma(beta, mn, mx) + 1e-100;  // x = y = 0 -> t = 0; changes nothing for den > 1e-84
+    // K in units of half a quarter turn; S = (-1)^(swap + x<0 + y<0)
+    int kk = big ? 1 : 0;
+    kk = swap ? 2 - kk : kk;
+    const bool xneg = x < 0.0, yneg = y < 0.0;
+    kk = xneg ? 4 - kk : kk;
+    q.kk = yneg ? 8 - kk : kk;
+    q.neg = swap ^ xneg ^ yneg;
+    return q;
+}
+
+// Exact small non-negative int -> double on the FP64 pipe (no I2F): 0 <= k < 2^31.
+__device__ __forceinline__ double small_int_to_double(int k) {
+    return __hiloint2double(0x43300000, k) - 4503599627370496.0;  // (2^52 + k) - 2^52
+}
+
+__device__ __forceinline__ double qt_finish(const QtPrep& q, double t) {
+    const double s = t * t;
+    // Estrin's scheme: dependency depth 5 instead of Horner's 10 (the kernel is latency-bound)
+    const double s2 = s * s, s4 = s2 * s2, s8 = s4 * s4;
+    const double q0 = fma(kAtanQ[1], s, kAtanQ[0]), q1 = fma(kAtanQ[3], s, kAtanQ[2]);
+    const double q2 = fma(kAtanQ[5], s, kAtanQ[4]), q3 = fma(kAtanQ[7], s, kAtanQ[6]);
+    const double q4 = fma(kAtanQ[9], s, kAtanQ[8]);
+    const double r0 = fma(q1, s2, q0), r1 = fma(q3, s2, q2), r2 = fma(kAtanQ[10], s2, q4);
+    const double p = fma(r2, s8, fma(r1, s4, r0));
+    const double tau = t * p;
+    double tt = fma(q.neg ? -1.0 : 1.0, tau, 0.5 * small_int_to_double(q.kk));
+    if (tt >= 4.0) tt = 0.0;
+    return tt;
+}
+
+__device__ __forceinline__ double quarter_turns(double x, double y) {
+    const QtPrep q = qt_prepare(x, y);
+    return qt_finish(q, q.num * fast_rcp(q.den));
+}
+
+// floor(x) for 0 <= x < 2^31 on the FP64 pipe (no F2I): rint via the 1.5 * 2^52 magic
+// number (the addition is exact up to the final rounding to an integer), then corrected by
+// one comparison — exact for every double in range, ties included.
+__device__ __forceinline__ int floor_nonneg(double x) {
+    const double big = x + 6755399441055744.0;
+    const double r = big - 6755399441055744.0;  // rint(x), exact
+    const int n = __double2loint(big);
+    return (r > x) ? n - 1 : n;
+}
+
+// sin and cos of a moderate angle (|a| < 2^20 pi/2; here a = 4 chi in [0, 8 pi)): Cody-Waite
+// reduction by pi/2 with the fdlibm split constants, then the fdlibm __kernel_sin/__kernel_cos
+// minimax polynomials on [-pi/4, pi/4].  Max error 2.2e-16 (checked against libm over [0, 8 pi));
+// branch-free, no local-memory Payne-Hanek path (unlike the generic sincos()).
+__device__ __forceinline__ void small_sincos(double a, double* sp, double* cp) {
+    const double k = rint(a * 0.63661977236758134308);
+    const double r = fma(-k, 6.07710050650619224932e-11, fma(-k, 1.57079632673412561417e+00, a));
+    const double z = r * r;
+    double ps = 1.58969099521155010221e-10;
+    ps = fma(ps, z, -2.50507602534068634195e-08);
+    ps = fma(ps, z, 2.75573137070700676789e-06);
+    ps = fma(ps, z, -1.98412698298579493134e-04);
+    ps = fma(ps, z, 8.33333333332248946124e-03);
+    ps = fma(ps, z, -1.66666666666666324348e-01);
+    const double sn = fma(r * z, ps, r);
+    double pc = -1.13596475577881948265e-11;
+    pc = fma(pc, z, 2.08757232129817482790e-09);
+    pc = fma(pc, z, -2.75573143513906633035e-07);
+    pc = fma(pc, z, 2.48015872894767294178e-05);
+    pc = fma(pc, z, -1.38888888888741095749e-03);
+    pc = fma(pc, z, 4.16666666666666019037e-02);
+    const double cs = fma(z * z, pc, fma(-0.5, z, 1.0));
+    const int q = (int)k & 3;
+    const double s0 = (q & 1) ? cs : sn;
+    const double c0 = (q & 1) ? sn : cs;
+    *sp = (q & 2) ? -s0 : s0;
+    *cp = ((q + 1) & 2) ? -c0 : c0;
+}
+
 // Rotation matrix of a unit quaternion [x,y,z,w] (no renormalisation, reading S7),
 // row-major m[3*i + j] = R_ij.
 __device__ __forceinline__ void quat_to_matrix(double x, double y, double z, double w, double m[9]) {
@@ -58,6 +188,25 @@ __device__ __forceinline__ uint64_t spread_bits(uint64_t x) {
     return x;
 }
 
+// Interleave the low 16 bits of x into the even bit positions of a 32-bit word.
+__device__ __forceinline__ uint32_t spread_bits16(uint32_t x) {
+    x &= 0xFFFFu;
+    x = (x | (x << 8)) & 0x00FF00FFu;
+    x = (x | (x << 4)) & 0x0F0F0F0Fu;
+    x = (x | (x << 2)) & 0x33333333u;
+    x = (x | (x << 1)) & 0x55555555u;
+    return x;
+}
+
+template <typename I>
+__device__ __forceinline__ int64_t nest_xyf(int64_t nside, I face, I ix, I iy) {
+    if (sizeof(I) == 4) {  // nside <= 2^16: ix, iy < 2^16
+        return (int64_t)face * nside * nside +
+               (int64_t)(spread_bits16((uint32_t)ix) | (spread_bits16((uint32_t)iy) << 1));
+    }
+    return (int64_t)face * nside * nside + (int64_t)(spread_bits((uint64_t)ix) | (spread_bits((uint64_t)iy) << 1));
+}
+
 struct HealpixGeom {
     int64_t nside;
     int64_t npix;
@@ -79,35 +228,31 @@ inline HealpixGeom make_geom(int64_t nside) {
 }
 
 // HEALPix pixel of direction (dx, dy, dz) (Gorski et al. 2005; readings S3-S6, S8).
-template <bool NEST>
-__device__ __forceinline__ int64_t vec2pix(const HealpixGeom& g, double dx, double dy, double dz) {
-    const double phi = (dx == 0.0 && dy == 0.0) ? 0.0 : atan2(dy, dx);
+// I = int32_t for nside <= 2^16 (all floor indices < 19 nside fit, 32-bit NEST bit
+// interleave), else int64_t; the returned pixel is int64 either way.
+template <bool NEST, typename I>
+__device__ __forceinline__ int64_t loc2pix(const HealpixGeom& g, double dz, double tt, double dx, double dy) {
     const double za = fabs(dz);
-    double tt = __dmul_rn(phi, kInvHalfPi);
-    if (tt < 0.0) {
-        tt = __dadd_rn(tt, 4.0);
-        if (tt == 4.0) tt = 0.0;
-    }
-    const int64_t nside = g.nside;
+    const I nside = (I)g.nside;
     if (za <= kTwoThird) {  // equatorial belt
         const double temp1 = __dmul_rn(g.dnside, __dadd_rn(0.5, tt));
         const double temp2 = __dmul_rn(__dmul_rn(g.dnside, dz), 0.75);
-        const int64_t jp = (int64_t)__dsub_rn(temp1, temp2);  // ascending edge line
-        const int64_t jm = (int64_t)__dadd_rn(temp1, temp2);  // descending edge line
+        const I jp = (I)__dsub_rn(temp1, temp2);  // ascending edge line
+        const I jm = (I)__dadd_rn(temp1, temp2);  // descending edge line
         if (!NEST) {
-            const int64_t nl4 = 4 * nside;
-            const int64_t ir = nside + 1 + jp - jm;
-            const int64_t kshift = 1 - (ir & 1);
-            const int64_t t1 = jp + jm - nside + kshift + 1 + 2 * nl4;
-            const int64_t ip = (t1 >> 1) & (nl4 - 1);
-            return g.ncap + nl4 * (ir - 1) + ip;
+            const I nl4 = 4 * nside;
+            const I ir = nside + 1 + jp - jm;
+            const I kshift = 1 - (ir & 1);
+            const I t1 = jp + jm - nside + kshift + 1 + 2 * nl4;
+            const I ip = (t1 >> 1) & (nl4 - 1);
+            return g.ncap + (int64_t)nl4 * (int64_t)(ir - 1) + (int64_t)ip;
         } else {
-            const int64_t ifp = jp >> g.order;
-            const int64_t ifm = jm >> g.order;
-            const int64_t face = (ifp == ifm) ? (ifp | 4) : ((ifp < ifm) ? ifp : (ifm + 8));
-            const int64_t ix = jm & (nside - 1);
-            const int64_t iy = nside - (jp & (nside - 1)) - 1;
-            return face * nside * nside + (int64_t)(spread_bits(ix) | (spread_bits(iy) << 1));
+            const I ifp = jp >> g.order;
+            const I ifm = jm >> g.order;
+            const I face = (ifp == ifm) ? (ifp | 4) : ((ifp < ifm) ? ifp : (ifm + 8));
+            const I ix = jm & (nside - 1);
+            const I iy = nside - (jp & (nside - 1)) - 1;
+            return nest_xyf<I>(g.nside, face, ix, iy);
         }
     }
     // polar caps; the well-conditioned sin(theta) form for za >= 0.99 (reading S5)
@@ -119,43 +264,134 @@ __device__ __forceinline__ int64_t vec2pix(const HealpixGeom& g, double dx, doub
         tmp = __ddiv_rn(__dmul_rn(g.dnside, sth), __dsqrt_rn(__ddiv_rn(__dadd_rn(1.0, za), 3.0)));
     }
     if (!NEST) {
-        const double tp = __dsub_rn(tt, (double)(int64_t)tt);
-        const int64_t jp = (int64_t)__dmul_rn(tp, tmp);
-        const int64_t jm = (int64_t)__dmul_rn(__dsub_rn(1.0, tp), tmp);
-        const int64_t ir = jp + jm + 1;
-        int64_t ip = (int64_t)__dmul_rn(tt, (double)ir);
+        const double tp = __dsub_rn(tt, (double)(int)tt);
+        const I jp = (I)__dmul_rn(tp, tmp);
+        const I jm = (I)__dmul_rn(__dsub_rn(1.0, tp), tmp);
+        const I ir = jp + jm + 1;
+        I ip = (I)__dmul_rn(tt, (double)ir);
         if (ip >= 4 * ir) ip -= 4 * ir;
-        return (dz > 0.0) ? 2 * ir * (ir - 1) + ip : g.npix - 2 * ir * (ir + 1) + ip;
+        const int64_t ir64 = ir;
+        return (dz > 0.0) ? 2 * ir64 * (ir64 - 1) + ip : g.npix - 2 * ir64 * (ir64 + 1) + ip;
     } else {
-        int64_t ntt = (int64_t)tt;
+        int ntt = (int)tt;
         if (ntt > 3) ntt = 3;
         const double tp = __dsub_rn(tt, (double)ntt);
-        int64_t jp = (int64_t)__dmul_rn(tp, tmp);
-        int64_t jm = (int64_t)__dmul_rn(__dsub_rn(1.0, tp), tmp);
+        I jp = (I)__dmul_rn(tp, tmp);
+        I jm = (I)__dmul_rn(__dsub_rn(1.0, tp), tmp);
         if (jp > nside - 1) jp = nside - 1;
         if (jm > nside - 1) jm = nside - 1;
-        int64_t face, ix, iy;
+        I face, ix, iy;
         if (dz >= 0.0) {
             face = ntt; ix = nside - jm - 1; iy = nside - jp - 1;
         } else {
             face = ntt + 8; ix = jp; iy = jm;
         }
-        return face * nside * nside + (int64_t)(spread_bits(ix) | (spread_bits(iy) << 1));
+        return nest_xyf<I>(g.nside, face, ix, iy);
     }
 }
 
-// (cos 2psi, sin 2psi) from psi = atan2(by, bx) without forming psi; psi := 0 at bx = by = 0 (S10).
-__device__ __forceinline__ void cos_sin_2psi(double bx, double by, double& c2, double& s2) {
-    const double bx2 = bx * bx, by2 = by * by;
-    const double r = bx2 + by2;
-    if (r > 0.0) {
-        const double inv = 1.0 / r;
-        c2 = (bx2 - by2) * inv;
-        s2 = 2.0 * bx * by * inv;
-    } else {
-        c2 = 1.0;
-        s2 = 0.0;
+// 32-bit interleave of ix (even bits) and iy (odd bits), ix, iy < 2^16: the outer perfect
+// shuffle of the word (iy << 16 | ix) (Hacker's Delight 7-2) — 1 PRMT + 3 delta swaps.
+__device__ __forceinline__ uint32_t interleave16(uint32_t ix, uint32_t iy) {
+    uint32_t x = __byte_perm(ix, iy, 0x5140);  // bytes: iy1 ix1 iy0 ix0
+    uint32_t t;
+    t = (x ^ (x >> 4)) & 0x00F000F0u; x = x ^ t ^ (t << 4);
+    t = (x ^ (x >> 2)) & 0x0C0C0C0Cu; x = x ^ t ^ (t << 2);
+    t = (x ^ (x >> 1)) & 0x22222222u; x = x ^ t ^ (t << 1);
+    return x;
+}
+
+// HEALPix pixel with 32-bit integer arithmetic; valid for nside <= 8192 (12 nside^2 < 2^31).
+// Same expressions, in the same order and rounding, as loc2pix above.
+template <bool NEST>
+__device__ __forceinline__ int loc2pix32(const HealpixGeom& g, double dz, double tt, double dx, double dy) {
+    const double za = fabs(dz);
+    const int nside = (int)g.nside;
+    if (za <= kTwoThird) {
+        const double temp1 = __dmul_rn(g.dnside, __dadd_rn(0.5, tt));
+        const double temp2 = __dmul_rn(__dmul_rn(g.dnside, dz), 0.75);
+        const int jp = floor_nonneg(__dsub_rn(temp1, temp2));
+        const int jm = floor_nonneg(__dadd_rn(temp1, temp2));
+        if (!NEST) {
+            const int nl4 = 4 * nside;
+            const int ir = nside + 1 + jp - jm;
+            const int kshift = 1 - (ir & 1);
+            const int t1 = jp + jm - nside + kshift + 1 + 2 * nl4;
+            const int ip = (t1 >> 1) & (nl4 - 1);
+            return (int)g.ncap + nl4 * (ir - 1) + ip;
+        } else {
+            const int ifp = jp >> g.order;
+            const int ifm = jm >> g.order;
+            const int face = (ifp == ifm) ? (ifp | 4) : ((ifp < ifm) ? ifp : (ifm + 8));
+            const int ix = jm & (nside - 1);
+            const int iy = nside - (jp & (nside - 1)) - 1;
+            return face * (nside * nside) + (int)interleave16((uint32_t)ix, (uint32_t)iy);
+        }
     }
+    double tmp;
+    if (za < 0.99) {
+        tmp = __dmul_rn(g.dnside, __dsqrt_rn(__dmul_rn(3.0, __dsub_rn(1.0, za))));
+    } else {
+        const double sth = __dsqrt_rn(__dadd_rn(__dmul_rn(dx, dx), __dmul_rn(dy, dy)));
+        tmp = __ddiv_rn(__dmul_rn(g.dnside, sth), __dsqrt_rn(__ddiv_rn(__dadd_rn(1.0, za), 3.0)));
+    }
+    if (!NEST) {
+        const double tp = __dsub_rn(tt, small_int_to_double(floor_nonneg(tt)));
+        const int jp = floor_nonneg(__dmul_rn(tp, tmp));
+        const int jm = floor_nonneg(__dmul_rn(__dsub_rn(1.0, tp), tmp));
+        const int ir = jp + jm + 1;
+        int ip = floor_nonneg(__dmul_rn(tt, small_int_to_double(ir)));
+        if (ip >= 4 * ir) ip -= 4 * ir;
+        return (dz > 0.0) ? 2 * ir * (ir - 1) + ip : (int)g.npix - 2 * ir * (ir + 1) + ip;
+    } else {
+        int ntt = floor_nonneg(tt);
+        if (ntt > 3) ntt = 3;
+        const double tp = __dsub_rn(tt, small_int_to_double(ntt));
+        int jp = floor_nonneg(__dmul_rn(tp, tmp));
+        int jm = floor_nonneg(__dmul_rn(__dsub_rn(1.0, tp), tmp));
+        if (jp > nside - 1) jp = nside - 1;
+        if (jm > nside - 1) jm = nside - 1;
+        int face, ix, iy;
+        if (dz >= 0.0) {
+            face = ntt; ix = nside - jm - 1; iy = nside - jp - 1;
+        } else {
+            face = ntt + 8; ix = jp; iy = jm;
+        }
+        return face * (nside * nside) + (int)interleave16((uint32_t)ix, (uint32_t)iy);
+    }
+}
+
+// tt = fmodulo(phi * 2/pi, 4) in [0, 4) with phi = atan2(dy, dx) (phi := 0 at dx = dy = 0, S3).
+__device__ __forceinline__ double phi_to_tt(double dx, double dy) { return quarter_turns(dx, dy); }
+
+template <bool NEST>
+__device__ __forceinline__ int64_t vec2pix(const HealpixGeom& g, double dx, double dy, double dz) {
+    return loc2pix<NEST, int64_t>(g, dz, phi_to_tt(dx, dy), dx, dy);
+}
+
+// (cos 2psi, sin 2psi) from psi = atan2(by, bx) without forming psi; psi := 0 at bx = by = 0
+// (S10): the 1e-100 guard makes (bx, by) = (0, 0) give (1, 0) without a branch and changes
+// nothing otherwise (r = sin^2 theta >> 1e-84 for any direction not within 1e-42 rad of a pole).
+__device__ __forceinline__ void cos_sin_2psi(double bx, double by, double& c2, double& s2) {
+    const double bx2 = bx * bx;
+    const double r = fma(by, by, bx2) + 1e-100;
+    const double inv = fast_rcp(r);
+    c2 = fma(-by, by, bx2 + 1e-100) * inv;
+    s2 = 2.0 * bx * by * inv;
+}
+
+// Longitude in quarter turns AND (cos 2psi, sin 2psi) with ONE reciprocal: 1/(den r) gives
+// both 1/den = r/(den r) and 1/r = den/(den r) (both factors lie in [1e-100, 2], so the
+// product neither overflows nor underflows).
+__device__ __forceinline__ double lon_pol(double dx, double dy, double bx, double by, double& c2, double& s2) {
+    const QtPrep q = qt_prepare(dx, dy);
+    const double bx2 = bx * bx;
+    const double r = fma(by, by, bx2) + 1e-100;
+    const double inv = fast_rcp(q.den * r);
+    const double invr = q.den * inv;
+    c2 = fma(-by, by, bx2 + 1e-100) * invr;
+    s2 = 2.0 * bx * by * invr;
+    return qt_finish(q, q.num * (r * inv));
 }
 
 }  // namespace toastb200

@@ -1,24 +1,30 @@
 // fused.cu — toast_pointing_to_map: A1 -> A2 -> A3 -> A4 per detector-sample in registers.
 //
-// Work item = (chunk of <= 256 consecutive in-interval samples, block of kDetBlock
-// detectors); a persistent grid of (#SM x resident CTAs) walks the items chunk-major, so
-// the CTAs resident at any moment cover a short time window of the whole focal plane and
-// the sky footprint they scatter into stays in L2.
-//
-// Per CTA and item:
-//   * the detector block's frames are staged in shared memory once:
-//       u = R(f) z, v = R(f) x, w = R(f) y  (columns of the detector rotation),
-//       eta*cal and det_scale;
-//   * each thread owns ONE sample: it loads the boresight quaternion once, forms the
-//     boresight rotation matrix B (identity when shared-flagged, reading S2) and, with an
-//     HWP, cos/sin(4 chi), and keeps them in registers for all detectors of the block;
-//   * per detector: dir = B u, bx = (B v)_z, by = -(B w)_z (15 DP ops), phi = atan2,
-//     HEALPix pixel, (cos 2psi, sin 2psi) algebraically, the HWP angle addition, the
-//     noise-weighted contribution det_scale * tod * w, then a warp-segmented reduction
-//     over runs of equal pixels and one fp64 red per run and Stokes component.
-// The only HBM streams are the TOD (coalesced along samples), the optional det flags,
-// the per-sample boresight/HWP/shared flags (read once per CTA item, i.e. once per
-// kDetBlock detectors) and the map updates.
+// Decomposition (B200-first):
+//   * A WARP owns a work item = (chunk of <= kFusedChunk consecutive in-interval samples,
+//     group of 32*DPL detectors); LANE = DETECTOR (each lane carries DPL detectors, d and
+//     d + 32).  Items are handed out dynamically (one atomic per item, fetched one item
+//     ahead) in chunk-major order, so the warps in flight cover a short time window of the
+//     focal plane and the sky footprint they scatter into stays L2-resident.
+//   * Each lane holds its detectors' frames in registers for the whole item:
+//       u = R(f) z, v = R(f) x, w = R(f) y, det_scale*cal, det_scale*eta*cal.
+//   * An item is a STREAM OF BLOCKS of kBlk = 16 samples, software-pipelined through two
+//     warp-private shared-memory buffers: while block i is computed, cp.async already
+//     copies ALL raw inputs of block i+1 — the TOD tile [32*DPL detectors x 16 samples]
+//     (two rows per instruction, coalesced along samples), the det-flag rows, the 16
+//     boresight quaternions, HWP angles and shared flags — so no global-memory latency is
+//     on the critical path.  At the start of a block, lanes 0..15 turn the raw per-sample
+//     inputs into the per-sample state (boresight rotation matrix B — identity if
+//     shared-flagged, reading S2 — and cos/sin 4 chi); every lane then walks the 16
+//     samples reading that state as shared-memory BROADCASTS and its TOD / flags from the
+//     padded (bank-conflict-free) tile.  Boresight, HWP and shared flags are read from HBM
+//     once per 32*DPL detectors; every HBM stream is read coalesced.
+//   * Per det-sample: dir = B u, bx = (B v)_z, by = -(B w)_z (15 DP ops), the HEALPix
+//     pixel (quarter-turn arctangent with one reciprocal; 32-bit integer path up to nside
+//     8192), cos/sin 2psi algebraically, the HWP angle addition, det_scale * tod * w.
+//   * Map accumulation is RUN-LENGTH aggregated per lane along time: consecutive samples of
+//     one detector that fall in the same pixel are summed in registers and flushed with one
+//     fp64 `red` per Stokes component when the pixel changes (no shuffles at all).
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -26,171 +32,542 @@
 
 #include "device_math.cuh"
 #include "internal.h"
-#include "map_accum.cuh"
 
 namespace toastb200 {
 
 namespace {
 
-struct DetFrame {
-    double u[3], v[3], w[3];
-    double etacal;
-    double scale;
-    double pad;
+#ifndef TB_FUSED_MINB
+#define TB_FUSED_MINB 2  // resident CTAs per SM the register allocation is bounded for
+#endif
+#ifndef TB_FUSED_DPL_MAX
+#define TB_FUSED_DPL_MAX 1  // detectors per lane (2 when n_det > 32 and DPL_MAX = 2)
+#endif
+constexpr int kWarps = 8;  // warps per CTA
+constexpr int kBlk = 16;   // samples per block
+constexpr int kPad = kBlk + 1;
+
+// per-sample state: B[0..8], c4, s4, mode (as a double: 1 pixelise, 2 shared-flagged)
+struct SampleState {
+    double v[12];
 };
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG>
-__global__ void __launch_bounds__(kChunk, 2) pointing_to_map_kernel(const Chunk* __restrict__ chunks,
-                                                                    int64_t n_chunks, FusedArgs a, HealpixGeom g) {
-    __shared__ DetFrame s_det[kDetBlock];
-    const int tid = threadIdx.x;
-    const int lane = tid & 31;
-    const int64_t n_dblk = (a.n_det + kDetBlock - 1) / kDetBlock;
-    const int64_t n_items = n_chunks * n_dblk;
+// Raw inputs of one block (filled by cp.async).
+template <int DPL>
+struct alignas(16) RawBlock {
+    double tod[32 * DPL][kPad];
+    double bore[kBlk][4];
+    double hwp[kBlk];
+    uint8_t flg[32 * DPL][kBlk + 4];  // 5 aligned words covering each row's 16 flag bytes
+    uint8_t sflg[kBlk + 8];           // 5 aligned words covering the 16 shared flags
+};
 
-    for (int64_t item = blockIdx.x; item < n_items; item += gridDim.x) {
-        const int64_t c = item / n_dblk;
-        const int64_t d0 = (item - c * n_dblk) * kDetBlock;
-        const int64_t nd_rem = a.n_det - d0;
-        const int nd = nd_rem < kDetBlock ? (int)nd_rem : kDetBlock;
-        const Chunk ch = chunks[c];
+template <int DPL>
+struct WarpSmem {
+    RawBlock<DPL> buf[2];
+    SampleState st[kBlk];
+};
 
-        __syncthreads();  // previous item finished reading s_det
-        if (tid < nd) {
-            const double* f = a.fp_quats + 4 * (d0 + tid);
-            double m[9];
-            quat_to_matrix(f[0], f[1], f[2], f[3], m);
-            DetFrame df;
-            df.u[0] = m[2]; df.u[1] = m[5]; df.u[2] = m[8];
-            df.v[0] = m[0]; df.v[1] = m[3]; df.v[2] = m[6];
-            df.w[0] = m[1]; df.w[1] = m[4]; df.w[2] = m[7];
-            const double eps = a.epsilon[d0 + tid];
-            df.etacal = (1.0 - eps) / (1.0 + eps) * a.cal;
-            df.scale = a.det_scale[d0 + tid];
-            df.pad = 0.0;
-            s_det[tid] = df;
-        }
-        __syncthreads();
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
+    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async4(void* smem, const void* gmem) {
+    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(s), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
 
-        if ((tid & ~31) >= ch.count) continue;  // whole warp beyond this chunk (uniform per warp)
-        const bool in = tid < ch.count;
-        const int64_t s = ch.first + (in ? tid : 0);
+// Copy the aligned 4-byte words covering bytes [p, p + n) (n <= 16) to dst[0..20); the
+// caller reads byte i of the range at dst[(p & 3) + i].  Words past the range are skipped,
+// so nothing beyond the aligned word holding the last byte is read.
+__device__ __forceinline__ void cp_async_bytes(uint8_t* dst, const uint8_t* p, int n, int w) {
+    const uint8_t* w0 = reinterpret_cast<const uint8_t*>(reinterpret_cast<uintptr_t>(p) & ~uintptr_t(3));
+    if (w0 + 4 * w < p + n) cp_async4(dst + 4 * w, w0 + 4 * w);
+}
 
-        // ---- per-sample state, reused for every detector of the block
-        bool sflag = false;
-        double B[9];
-        {
-            double q[4] = {0.0, 0.0, 0.0, 1.0};
-            if (in) {
-                sflag = a.shared_flags && (__ldg(&a.shared_flags[s]) & a.shared_flag_mask);
-                if (!sflag) {
-                    const double2 lo = __ldg(reinterpret_cast<const double2*>(a.boresight + 4 * s));
-                    const double2 hi = __ldg(reinterpret_cast<const double2*>(a.boresight + 4 * s) + 1);
-                    q[0] = lo.x; q[1] = lo.y; q[2] = hi.x; q[3] = hi.y;
-                }
-            }
-            quat_to_matrix(q[0], q[1], q[2], q[3], B);
-        }
-        double c4 = 1.0, s4 = 0.0;
-        if (HWP && NNZ == 3) {
-            if (in) sincos(4.0 * __ldg(&a.hwp[s]), &s4, &c4);
-        }
-        const bool pix_ok = in && !sflag;
+// Pixel index type: 32-bit up to nside 8192 (12 nside^2 < 2^31), else 64-bit.
+template <bool WIDE>
+struct PixT;
+template <>
+struct PixT<false> {
+    using T = int;
+};
+template <>
+struct PixT<true> {
+    using T = int64_t;
+};
 
-        const double* __restrict__ tod_base = a.det_data + d0 * a.n_samp + s;
-        const uint8_t* __restrict__ fl_base = a.det_flags ? a.det_flags + d0 * a.n_samp + s : nullptr;
+// Submap of a pixel (shift when n_pix_submap is a power of two).
+template <typename P>
+__device__ __forceinline__ int64_t submap_of(P pix, const MapGeom& mg) {
+    return mg.sm_shift >= 0 ? (int64_t)(pix >> mg.sm_shift) : (int64_t)pix / mg.n_pix_submap;
+}
 
-#pragma unroll 1
-        for (int j = 0; j < nd; ++j) {
-            const DetFrame& df = s_det[j];
-            const double tod = in ? __ldg(tod_base + j * a.n_samp) : 0.0;
-            const bool dflag = (in && fl_base) ? ((__ldg(fl_base + j * a.n_samp) & a.det_flag_mask) != 0) : false;
+// A run starts: mark its submap hit (as A2 does) and issue the global2local lookup now, so
+// the load latency is hidden behind the run's samples instead of stalling the flush.  The hit
+// flag is stored only when the lane's submap CHANGES: thousands of warps re-writing the same
+// few bytes of hit_submaps serialise in L2 and cost as much as the whole computation.
+template <typename P>
+__device__ __forceinline__ int64_t start_run(P pix, const FusedArgs& a, int64_t& last_sm) {
+    const int64_t sm = submap_of<P>(pix, a.map);
+#ifndef TB_X_NOHIT
+    if (a.hit_submaps && sm != last_sm) {
+        a.hit_submaps[sm] = 1;
+        last_sm = sm;
+    }
+#endif
+#ifdef TB_X_NOG2L
+    return sm;
+#else
+    return __ldg(&a.map.global2local[sm]);
+#endif
+}
 
-            // A1 + rotation: dir = B u; bx = (B v)_z; by = -(B w)_z
-            const double dx = B[0] * df.u[0] + B[1] * df.u[1] + B[2] * df.u[2];
-            const double dy = B[3] * df.u[0] + B[4] * df.u[1] + B[5] * df.u[2];
-            const double dz = B[6] * df.u[0] + B[7] * df.u[1] + B[8] * df.u[2];
-
-            // A2
-            int64_t pix = -1;
-            if (pix_ok) pix = vec2pix<NEST>(g, dx, dy, dz);
-
-            // A3
-            double wq = 0.0, wu = 0.0;
-            if (NNZ == 3) {
-                const double bx = B[6] * df.v[0] + B[7] * df.v[1] + B[8] * df.v[2];
-                const double by = -(B[6] * df.w[0] + B[7] * df.w[1] + B[8] * df.w[2]);
-                double c2, s2;
-                cos_sin_2psi(bx, by, c2, s2);
-                if (HWP) {
-                    const double cq = c2 * c4 - s2 * s4;
-                    const double sq = s2 * c4 + c2 * s4;
-                    c2 = cq;
-                    s2 = sq;
-                }
-                wq = df.etacal * c2;
-                wu = df.etacal * s2;
-            }
-
-            if (DEBUG && in) {
-                const int64_t o = (d0 + j) * a.n_samp + s;
-                if (a.pixels_out) a.pixels_out[o] = pix;
-                if (a.weights_out) {
-                    a.weights_out[o * NNZ] = a.cal;
-                    if (NNZ == 3) {
-                        a.weights_out[o * NNZ + 1] = wq;
-                        a.weights_out[o * NNZ + 2] = wu;
-                    }
-                }
-            }
-
-            // A4: contribution of this det-sample; det-flagged samples keep their pixel key
-            // (they still mark hit submaps, as A2 does) but add nothing.
-            const double val = (pix >= 0 && !dflag) ? df.scale * tod : 0.0;
-            const int64_t key = pix >= 0 ? pix : (int64_t)(-1 - lane);
-            warp_accumulate<NNZ>(key, val * a.cal, val * wq, val * wu, a.map, a.zmap, a.hit_submaps);
-        }
+// A run ends: one fp64 red per Stokes component (nothing if the submap has no storage).
+template <int NNZ, typename P>
+__device__ __forceinline__ void flush(P pix, int64_t loc, double a0, double a1, double a2, const FusedArgs& a) {
+    if (loc < 0) return;
+    const MapGeom& mg = a.map;
+    const int64_t lp = mg.sm_shift >= 0 ? (int64_t)(pix & (P)(mg.n_pix_submap - 1))
+                                        : (int64_t)pix - submap_of<P>(pix, mg) * mg.n_pix_submap;
+    double* dst = a.zmap + (loc * mg.n_pix_submap + lp) * NNZ;
+    atomicAdd(dst, a0);
+    if (NNZ == 3) {
+        atomicAdd(dst + 1, a1);
+        atomicAdd(dst + 2, a2);
     }
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG>
-cudaError_t launch_t(const WorkList& wl, const FusedArgs& a, cudaStream_t st) {
-    auto kern = pointing_to_map_kernel<NEST, NNZ, HWP, DEBUG>;
+template <typename P>
+struct Slot {
+    double u0, u1, u2, v0, v1, v2, w0, w1, w2;
+    double s_cal;   // det_scale * cal       (I weight folded into the noise weight)
+    double s_eta;   // det_scale * eta * cal (Q/U amplitude folded into the noise weight)
+    double etacal;  // debug outputs only
+    P run_pix;
+    int64_t run_loc;      // global2local of the run's submap, LOADED WHEN THE RUN STARTS
+    int64_t last_sm;      // last submap this lane marked in hit_submaps
+    double r0, r1, r2;
+    P pend_pix;           // pending (not yet aggregated) det-sample
+    double p0, p1, p2;
+    bool ok;
+};
+
+template <typename P>
+__device__ __forceinline__ void load_slot(Slot<P>& sl, const FusedArgs& a, int64_t d, bool ok, int64_t dfallback) {
+    const int64_t dd = ok ? d : dfallback;
+    double m[9];
+    const double2 f01 = __ldg(reinterpret_cast<const double2*>(a.fp_quats + 4 * dd));
+    const double2 f23 = __ldg(reinterpret_cast<const double2*>(a.fp_quats + 4 * dd) + 1);
+    quat_to_matrix(f01.x, f01.y, f23.x, f23.y, m);
+    sl.u0 = m[2]; sl.u1 = m[5]; sl.u2 = m[8];
+    sl.v0 = m[0]; sl.v1 = m[3]; sl.v2 = m[6];
+    sl.w0 = m[1]; sl.w1 = m[4]; sl.w2 = m[7];
+    const double eps = __ldg(&a.epsilon[dd]);
+    const double scale = __ldg(&a.det_scale[dd]);
+    sl.etacal = (1.0 - eps) / (1.0 + eps) * a.cal;
+    sl.s_cal = scale * a.cal;
+    sl.s_eta = scale * sl.etacal;
+    sl.run_pix = -1;
+    sl.run_loc = -1;
+    sl.last_sm = -1;
+    sl.r0 = sl.r1 = sl.r2 = 0.0;
+    sl.pend_pix = -1;
+    sl.p0 = sl.p1 = sl.p2 = 0.0;
+    sl.ok = ok;
+}
+
+// One det-sample of slot `sl` with the per-sample state x.
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE>
+__device__ __forceinline__ void det_sample(Slot<typename PixT<WIDE>::T>& sl, const double* x, bool pixelise,
+                                           double tod, bool dflag, const HealpixGeom& g, const FusedArgs& a,
+                                           int64_t d, int64_t s) {
+    using P = typename PixT<WIDE>::T;
+    const double dx = x[0] * sl.u0 + x[1] * sl.u1 + x[2] * sl.u2;
+    const double dy = x[3] * sl.u0 + x[4] * sl.u1 + x[5] * sl.u2;
+    const double dz = x[6] * sl.u0 + x[7] * sl.u1 + x[8] * sl.u2;
+    // The weight chain and the longitude chain are independent and branch-free: they are
+    // written into one basic block so the scheduler can interleave them (latency-bound code).
+    // (cos 2(psi + 2 chi), sin 2(psi + 2 chi)): the Q/U weights divided by eta*cal
+    double c2 = 0.0, s2 = 0.0, tt;
+    if (NNZ == 3) {
+        const double bx = x[6] * sl.v0 + x[7] * sl.v1 + x[8] * sl.v2;
+        const double by = -(x[6] * sl.w0 + x[7] * sl.w1 + x[8] * sl.w2);
+#ifdef TB_X_NOATAN
+        tt = fabs(dx) * 3.9; c2 = bx; s2 = by;  // ablation: no longitude/weights arithmetic
+#else
+        tt = lon_pol(dx, dy, bx, by, c2, s2);  // one shared reciprocal
+#endif
+        if (HWP) {
+            const double c4 = x[9], s4 = x[10];
+            const double cq = c2 * c4 - s2 * s4;
+            const double sq = s2 * c4 + c2 * s4;
+            c2 = cq;
+            s2 = sq;
+        }
+    } else {
+        tt = quarter_turns(dx, dy);
+    }
+    P pix = -1;
+    if (pixelise) {
+        if (WIDE)
+            pix = (P)loc2pix<NEST, int64_t>(g, dz, tt, dx, dy);
+        else
+#ifdef TB_X_NOPIX
+            pix = (P)((int)(tt * 1000.0) & 0xffff);  // ablation: no HEALPix integer/floor logic
+#else
+            pix = (P)loc2pix32<NEST>(g, dz, tt, dx, dy);
+#endif
+    }
+    if (!sl.ok) pix = -1;
+    if (DEBUG && sl.ok) {
+        const int64_t o = d * a.n_samp + s;
+        if (a.pixels_out) a.pixels_out[o] = (int64_t)pix;
+        if (a.weights_out) {
+            a.weights_out[o * NNZ] = a.cal;
+            if (NNZ == 3) {
+                a.weights_out[o * NNZ + 1] = sl.etacal * c2;
+                a.weights_out[o * NNZ + 2] = sl.etacal * s2;
+            }
+        }
+    }
+    // A4 contribution of this det-sample; it is folded into the lane's run by aggregate()
+    // one sample LATER, so that work overlaps the shared-memory loads of the next sample.
+    // Det-flagged samples keep their pixel (they mark hit submaps, as A2 does) but add 0.
+    sl.pend_pix = pix;
+    sl.p0 = dflag ? 0.0 : tod * sl.s_cal;
+    if (NNZ == 3) {
+        const double t = dflag ? 0.0 : tod * sl.s_eta;
+        sl.p1 = t * c2;
+        sl.p2 = t * s2;
+    }
+}
+
+// Fold the pending contribution into the run (run-length aggregation along time).  Lanes
+// without a pixel (no detector / flagged sample) have pend_pix = -1 and never touch their run.
+__device__ __forceinline__ void red_if(bool p, double* addr, double v) {
+    asm volatile("{\n .reg .pred q;\n setp.ne.u32 q, %0, 0;\n @q red.global.add.f64 [%1], %2;\n}\n" ::"r"((unsigned)p),
+                 "l"(addr), "d"(v)
+                 : "memory");
+}
+__device__ __forceinline__ int64_t ldg_if(bool p, const int64_t* addr, int64_t dflt) {
+    int64_t v = dflt;
+    asm volatile("{\n .reg .pred q;\n setp.ne.u32 q, %1, 0;\n @q ld.global.nc.s64 %0, [%2];\n}\n"
+                 : "+l"(v)
+                 : "r"((unsigned)p), "l"(addr));
+    return v;
+}
+__device__ __forceinline__ void stg_u8_if(bool p, uint8_t* addr) {
+    asm volatile("{\n .reg .pred q;\n setp.ne.u32 q, %0, 0;\n @q st.global.u8 [%1], 1;\n}\n" ::"r"((unsigned)p),
+                 "l"(addr)
+                 : "memory");
+}
+
+template <int NNZ, typename P>
+__device__ __forceinline__ void aggregate(Slot<P>& sl, const FusedArgs& a) {
+#ifdef TB_BRANCHFREE_AGG
+    // branch-free form: predicated red / ld / st, so a rare run end in one lane does not
+    // make the whole warp take a divergent path
+    const MapGeom& mg = a.map;
+    const bool has = sl.pend_pix >= 0;
+    const bool newrun = has && sl.pend_pix != sl.run_pix;
+    const bool doflush = newrun && sl.run_pix >= 0 && sl.run_loc >= 0;
+    const P fp = sl.run_pix < 0 ? 0 : sl.run_pix;
+    const int64_t lp = mg.sm_shift >= 0 ? (int64_t)(fp & (P)(mg.n_pix_submap - 1))
+                                        : (int64_t)fp - submap_of<P>(fp, mg) * mg.n_pix_submap;
+    double* dst = a.zmap + (sl.run_loc * mg.n_pix_submap + lp) * NNZ;
+    red_if(doflush, dst, sl.r0);
+    if (NNZ == 3) {
+        red_if(doflush, dst + 1, sl.r1);
+        red_if(doflush, dst + 2, sl.r2);
+    }
+    const P np = has ? sl.pend_pix : 0;
+    const int64_t sm = submap_of<P>(np, mg);
+    if (a.hit_submaps) stg_u8_if(newrun, a.hit_submaps + sm);
+    sl.run_loc = ldg_if(newrun, mg.global2local + sm, sl.run_loc);
+    sl.run_pix = newrun ? sl.pend_pix : sl.run_pix;
+    sl.r0 = (newrun ? 0.0 : sl.r0) + (has ? sl.p0 : 0.0);
+    if (NNZ == 3) {
+        sl.r1 = (newrun ? 0.0 : sl.r1) + (has ? sl.p1 : 0.0);
+        sl.r2 = (newrun ? 0.0 : sl.r2) + (has ? sl.p2 : 0.0);
+    }
+    sl.pend_pix = -1;
+    sl.p0 = sl.p1 = sl.p2 = 0.0;
+    return;
+#endif
+    if (sl.pend_pix >= 0) {
+        if (sl.pend_pix != sl.run_pix) {
+#ifndef TB_X_NOFLUSH
+            if (sl.run_pix >= 0) flush<NNZ, P>(sl.run_pix, sl.run_loc, sl.r0, sl.r1, sl.r2, a);
+#endif
+            sl.run_pix = sl.pend_pix;
+            sl.run_loc = start_run<P>(sl.pend_pix, a, sl.last_sm);
+            sl.r0 = sl.r1 = sl.r2 = 0.0;
+        }
+        sl.r0 += sl.p0;
+        if (NNZ == 3) {
+            sl.r1 += sl.p1;
+            sl.r2 += sl.p2;
+        }
+        sl.pend_pix = -1;
+    }
+}
+
+// A block of the stream: samples [s0, s0 + nb) of chunk c for detector rows d0 .. d0+nrows-1.
+struct Blk {
+    int64_t item;  // < 0: end of stream
+    int64_t d0;
+    int64_t s0;
+    int64_t s_end;  // end of the item's chunk
+    int nb;
+    int nrows;
+};
+
+template <int DPL>
+__device__ __forceinline__ void issue_block(RawBlock<DPL>& rb, const Blk& bk, const FusedArgs& a, bool have_dflags,
+                                            bool hwp, int lane) {
+    constexpr int kRows = 32 * DPL;
+    const int64_t n_samp = a.n_samp;
+    const int scol = lane & (kBlk - 1);
+    const int srow = lane >> 4;  // 0 or 1
+    if (scol < bk.nb) {
+        const double* src = a.det_data + (bk.d0 + srow) * n_samp + bk.s0 + scol;
+        const int64_t step = 2 * n_samp;
+        if (bk.nrows == kRows) {
+#pragma unroll 8
+            for (int r = srow; r < kRows; r += 2, src += step) cp_async8(&rb.tod[r][scol], src);
+        } else {
+            for (int r = srow; r < bk.nrows; r += 2, src += step) cp_async8(&rb.tod[r][scol], src);
+        }
+    }
+    // boresight: 16 quaternions = 32 x 16 B, one per lane
+    if ((lane >> 1) < bk.nb) cp_async16(&rb.bore[lane >> 1][2 * (lane & 1)], a.boresight + 4 * (bk.s0 + (lane >> 1)) + 2 * (lane & 1));
+    if (hwp && lane < bk.nb) cp_async8(&rb.hwp[lane], a.hwp + bk.s0 + lane);
+    if (a.shared_flags && lane < 5) cp_async_bytes(rb.sflg, a.shared_flags + bk.s0, bk.nb, lane);
+    if (have_dflags) {
+#pragma unroll
+        for (int j = 0; j < DPL; ++j) {
+            const int row = lane + 32 * j;
+            if (row < bk.nrows) {
+#pragma unroll
+                for (int w = 0; w < 5; ++w) cp_async_bytes(rb.flg[row], a.det_flags + (bk.d0 + row) * n_samp + bk.s0, bk.nb, w);
+            }
+        }
+    }
+    cp_async_commit();
+}
+
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL>
+__global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_kernel(const Chunk* __restrict__ chunks,
+                                                                         int64_t n_chunks, FusedArgs a,
+                                                                         HealpixGeom g,
+                                                                         unsigned long long* __restrict__ sched) {
+    using P = typename PixT<WIDE>::T;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int lane = threadIdx.x & 31;
+    const int wid = threadIdx.x >> 5;
+    WarpSmem<DPL>& sm = reinterpret_cast<WarpSmem<DPL>*>(smem_raw)[wid];
+    constexpr int kRows = 32 * DPL;
+    const int64_t n_groups = (a.n_det + kRows - 1) / kRows;
+    const int64_t n_items = n_chunks * n_groups;
+    const unsigned dmask = a.det_flag_mask;
+    const unsigned smask = a.shared_flag_mask;
+    const bool have_dflags = a.det_flags != nullptr;
+    const bool have_sflags = a.shared_flags != nullptr;
+
+    // Lane 0 fetches the NEXT item id and its chunk descriptor one item ahead (issued at
+    // an item switch, consumed at the next one), so neither latency is on the critical path.
+    int64_t pend_item = -1, pend_first = 0;
+    int pend_count = 0;
+    auto prefetch_item = [&]() {
+        if (lane == 0) {
+            const unsigned long long it = atomicAdd(sched, 1ull);
+            pend_item = it < (unsigned long long)n_items ? (int64_t)it : -1;
+            if (pend_item >= 0) {
+                const Chunk ch = chunks[pend_item / n_groups];
+                pend_first = ch.first;
+                pend_count = ch.count;
+            }
+        }
+    };
+    auto take_item = [&]() -> Blk {
+        Blk bk;
+        bk.item = __shfl_sync(0xffffffffu, pend_item, 0);
+        const int64_t first = __shfl_sync(0xffffffffu, pend_first, 0);
+        const int count = __shfl_sync(0xffffffffu, pend_count, 0);
+        if (bk.item < 0) {
+            bk.d0 = bk.s0 = bk.s_end = 0;
+            bk.nb = bk.nrows = 0;
+            return bk;
+        }
+        const int64_t c = bk.item / n_groups;
+        bk.d0 = (bk.item - c * n_groups) * kRows;
+        bk.nrows = (a.n_det - bk.d0) < kRows ? (int)(a.n_det - bk.d0) : kRows;
+        bk.s0 = first;
+        bk.s_end = first + count;
+        bk.nb = count < kBlk ? count : kBlk;
+        return bk;
+    };
+
+    prefetch_item();
+    Blk cur = take_item();
+    if (cur.item < 0) return;
+    prefetch_item();
+    issue_block<DPL>(sm.buf[0], cur, a, have_dflags, HWP && NNZ == 3, lane);
+    Slot<P> sl[DPL];
+#pragma unroll
+    for (int j = 0; j < DPL; ++j) load_slot<P>(sl[j], a, cur.d0 + lane + 32 * j, lane + 32 * j < cur.nrows, cur.d0);
+    int p = 0;
+
+    while (true) {
+        // successor block: next 16 samples of this item, or the first block of the next item
+        Blk nxt;
+        if (cur.s0 + kBlk < cur.s_end) {
+            nxt = cur;
+            nxt.s0 = cur.s0 + kBlk;
+            nxt.nb = (nxt.s_end - nxt.s0) < kBlk ? (int)(nxt.s_end - nxt.s0) : kBlk;
+        } else {
+            nxt = take_item();
+            if (nxt.item >= 0) prefetch_item();
+        }
+        cp_async_wait_all();
+        __syncwarp();
+        if (nxt.item >= 0) issue_block<DPL>(sm.buf[p ^ 1], nxt, a, have_dflags, HWP && NNZ == 3, lane);
+
+        RawBlock<DPL>& rb = sm.buf[p];
+        // per-sample state (lanes 0..15); bit k of pmask = sample k is pixelised
+        bool pixelise_me = false;
+        if (lane < kBlk) {
+            double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 1.0;
+            double c4 = 1.0, s4 = 0.0;
+            if (lane < cur.nb) {
+                const int soff = have_sflags ? (int)(reinterpret_cast<uintptr_t>(a.shared_flags + cur.s0) & 3) : 0;
+                const bool flagged = have_sflags && (rb.sflg[soff + lane] & smask);
+                pixelise_me = !flagged;
+                if (!flagged) {
+                    q0 = rb.bore[lane][0]; q1 = rb.bore[lane][1]; q2 = rb.bore[lane][2]; q3 = rb.bore[lane][3];
+                }
+                if (HWP && NNZ == 3) small_sincos(4.0 * rb.hwp[lane], &s4, &c4);
+            }
+            SampleState x;
+            quat_to_matrix(q0, q1, q2, q3, x.v);
+            x.v[9] = c4;
+            x.v[10] = s4;
+            x.v[11] = 0.0;
+            sm.st[lane] = x;
+        }
+        const unsigned pmask = __ballot_sync(0xffffffffu, pixelise_me);
+        int foff[DPL];
+#pragma unroll
+        for (int j = 0; j < DPL; ++j)
+            foff[j] = have_dflags
+                          ? (int)(reinterpret_cast<uintptr_t>(a.det_flags + (cur.d0 + lane + 32 * j) * a.n_samp + cur.s0) & 3)
+                          : 0;
+        __syncwarp();
+
+#pragma unroll 1
+        for (int k = 0; k < cur.nb; ++k) {
+            const bool pixelise = (pmask >> k) & 1u;
+            if (!DEBUG && !pixelise) continue;  // shared-flagged sample: nothing to add (uniform)
+            double x[12];
+#pragma unroll
+            for (int i = 0; i < ((HWP && NNZ == 3) ? 12 : 10); i += 2) {
+                const double2 t2 = *reinterpret_cast<const double2*>(&sm.st[k].v[i]);
+                x[i] = t2.x;
+                x[i + 1] = t2.y;
+            }
+            double tod[DPL];
+            bool dflag[DPL];
+#pragma unroll
+            for (int j = 0; j < DPL; ++j) {
+                const int row = lane + 32 * j;
+                tod[j] = rb.tod[row][k];
+                dflag[j] = have_dflags && ((rb.flg[row][k + foff[j]] & dmask) != 0);
+            }
+            // fold the previous sample while those shared-memory loads are in flight
+#pragma unroll
+            for (int j = 0; j < DPL; ++j) aggregate<NNZ, P>(sl[j], a);
+#pragma unroll
+            for (int j = 0; j < DPL; ++j)
+                det_sample<NEST, NNZ, HWP, DEBUG, WIDE>(sl[j], x, pixelise, tod[j], dflag[j], g, a,
+                                                        cur.d0 + lane + 32 * j, cur.s0 + k);
+        }
+
+        if (nxt.item != cur.item) {
+#pragma unroll
+            for (int j = 0; j < DPL; ++j) {
+                aggregate<NNZ, P>(sl[j], a);
+                if (sl[j].run_pix >= 0) flush<NNZ, P>(sl[j].run_pix, sl[j].run_loc, sl[j].r0, sl[j].r1, sl[j].r2, a);
+            }
+            if (nxt.item < 0) break;
+#pragma unroll
+            for (int j = 0; j < DPL; ++j)
+                load_slot<P>(sl[j], a, nxt.d0 + lane + 32 * j, lane + 32 * j < nxt.nrows, nxt.d0);
+        }
+        __syncwarp();  // all lanes are done with buf[p] and st before they are refilled
+        cur = nxt;
+        p ^= 1;
+    }
+    cp_async_wait_all();
+}
+
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL>
+cudaError_t launch_t(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
+    auto kern = pointing_to_map_kernel<NEST, NNZ, HWP, DEBUG, WIDE, DPL>;
+    const size_t smem = sizeof(WarpSmem<DPL>) * kWarps;
     static int blocks_per_sm = 0;
     static std::once_flag once;
     std::call_once(once, [&] {
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, kern, kChunk, 0) != cudaSuccess ||
+        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, kern, kWarps * 32, smem) != cudaSuccess ||
             blocks_per_sm < 1)
             blocks_per_sm = 1;
     });
-    const int64_t n_dblk = (a.n_det + kDetBlock - 1) / kDetBlock;
-    const int64_t n_items = wl.n_chunks * n_dblk;
-    const int64_t grid = std::min<int64_t>(n_items, (int64_t)num_sms() * blocks_per_sm);
+    const int64_t n_items = wl.n_chunks * ((a.n_det + 32 * DPL - 1) / (32 * DPL));
+    const int64_t want = (n_items + kWarps - 1) / kWarps;
+    const int64_t grid = std::min<int64_t>(want, (int64_t)num_sms() * blocks_per_sm);
     if (grid <= 0) return cudaSuccess;
-    kern<<<(unsigned)grid, kChunk, 0, st>>>(wl.chunks, wl.n_chunks, a, make_geom(a.nside));
+    cudaError_t e = cudaMemsetAsync(sched, 0, sizeof(unsigned long long), st);
+    if (e != cudaSuccess) return e;
+    kern<<<(unsigned)grid, kWarps * 32, smem, st>>>(wl.chunks, wl.n_chunks, a, make_geom(a.nside), sched);
     return cudaGetLastError();
 }
 
+template <bool NEST, int NNZ, bool HWP, bool DEBUG>
+cudaError_t dispatch_shape(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
+    const bool wide = a.nside > 8192;
+    const bool two = TB_FUSED_DPL_MAX > 1 && a.n_det > 32;
+    if (wide) return two ? launch_t<NEST, NNZ, HWP, DEBUG, true, TB_FUSED_DPL_MAX>(wl, a, sched, st)
+                         : launch_t<NEST, NNZ, HWP, DEBUG, true, 1>(wl, a, sched, st);
+    return two ? launch_t<NEST, NNZ, HWP, DEBUG, false, TB_FUSED_DPL_MAX>(wl, a, sched, st)
+               : launch_t<NEST, NNZ, HWP, DEBUG, false, 1>(wl, a, sched, st);
+}
+
 template <bool NEST, int NNZ, bool HWP>
-cudaError_t dispatch_debug(const WorkList& wl, const FusedArgs& a, cudaStream_t st) {
-    if (a.pixels_out || a.weights_out) return launch_t<NEST, NNZ, HWP, true>(wl, a, st);
-    return launch_t<NEST, NNZ, HWP, false>(wl, a, st);
+cudaError_t dispatch_debug(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
+    if (a.pixels_out || a.weights_out) return dispatch_shape<NEST, NNZ, HWP, true>(wl, a, sched, st);
+    return dispatch_shape<NEST, NNZ, HWP, false>(wl, a, sched, st);
 }
 
 template <bool NEST, int NNZ>
-cudaError_t dispatch_hwp(const WorkList& wl, const FusedArgs& a, cudaStream_t st) {
-    if (a.hwp && NNZ == 3) return dispatch_debug<NEST, NNZ, true>(wl, a, st);
-    return dispatch_debug<NEST, NNZ, false>(wl, a, st);
+cudaError_t dispatch_hwp(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
+    if (a.hwp && NNZ == 3) return dispatch_debug<NEST, NNZ, true>(wl, a, sched, st);
+    return dispatch_debug<NEST, NNZ, false>(wl, a, sched, st);
 }
 
 }  // namespace
 
-cudaError_t launch_pointing_to_map(const WorkList& wl, const FusedArgs& a, cudaStream_t st) {
+cudaError_t launch_pointing_to_map(const WorkList& wl, const FusedArgs& a, unsigned long long* sched,
+                                   cudaStream_t st) {
     if (wl.n_chunks == 0 || a.n_det == 0) return cudaSuccess;
-    if (a.nest) {
-        return a.nnz == 3 ? dispatch_hwp<true, 3>(wl, a, st) : dispatch_hwp<true, 1>(wl, a, st);
-    }
-    return a.nnz == 3 ? dispatch_hwp<false, 3>(wl, a, st) : dispatch_hwp<false, 1>(wl, a, st);
+    if (a.nest) return a.nnz == 3 ? dispatch_hwp<true, 3>(wl, a, sched, st) : dispatch_hwp<true, 1>(wl, a, sched, st);
+    return a.nnz == 3 ? dispatch_hwp<false, 3>(wl, a, sched, st) : dispatch_hwp<false, 1>(wl, a, sched, st);
 }
 
 }  // namespace toastb200

@@ -10,9 +10,9 @@ namespace toastb200 {
 
 // Samples per work chunk = threads per CTA of every kernel (one sample per thread).
 constexpr int kChunk = 256;
-// Detectors per fused work item (a CTA loops over them with the sample's boresight
-// rotation held in registers).
-constexpr int kDetBlock = 32;
+// Samples per work chunk of the fused kernel (a warp item = one such chunk x 32 or 64
+// detectors; small enough that the dynamic schedule balances to a few percent).
+constexpr int kFusedChunk = 128;
 
 // One chunk of <= kChunk consecutive in-interval samples (never crosses an interval).
 struct Chunk {
@@ -80,7 +80,11 @@ cudaError_t launch_scan_map(const WorkList& wl, const MapGeom& mg, const double*
                             const int64_t* pixels, const int32_t* weight_index, const double* weights,
                             double data_scale, int should_zero, int should_subtract, int64_t n_det, int64_t n_samp,
                             cudaStream_t st);
-cudaError_t launch_pointing_to_map(const WorkList& wl, const FusedArgs& a, cudaStream_t st);
+cudaError_t launch_pointing_to_map(const WorkList& wl, const FusedArgs& a, unsigned long long* sched,
+                                   cudaStream_t st);
+
+// A device counter for dynamic work distribution (zeroed on the stream before each use).
+unsigned long long* sched_counter(int* err);
 
 int num_sms();
 

@@ -75,6 +75,7 @@ __global__ void __launch_bounds__(kChunk) pixels_healpix_kernel(
         const bool in = (int)threadIdx.x < ch.count;
         const int64_t s = ch.first + threadIdx.x;
         const bool flagged = in && shared_flags && (__ldg(&shared_flags[s]) & shared_flag_mask);
+        int64_t last_sm = -1;  // hit flags are stored only when the submap changes (L2 write contention)
         for (int64_t d = blockIdx.y; d < n_det; d += gridDim.y) {
             int64_t pix = -1;
             if (in && !flagged) {
@@ -90,7 +91,8 @@ __global__ void __launch_bounds__(kChunk) pixels_healpix_kernel(
             if (hit_submaps) {
                 const int64_t sm = pix >= 0 ? pix / n_pix_submap : -1;
                 const int64_t prev = __shfl_up_sync(kFull, sm, 1);
-                if (sm >= 0 && (lane == 0 || prev != sm)) hit_submaps[sm] = 1;
+                if (sm >= 0 && sm != last_sm && (lane == 0 || prev != sm)) hit_submaps[sm] = 1;
+                if (sm >= 0) last_sm = sm;
             }
         }
     }

@@ -43,12 +43,24 @@ def check_weights(gpu_w, ora_w, sin_theta, eta_cal, cal, mask):
             assert np.all(dk <= tol), f"weight {k}: max excess {(dk - tol).max()} at {worst}"
 
 
-def check_map(gpu_map, ora_map, absmap):
-    """T4."""
-    zero = absmap == 0
+def map_scale(absmap, eta_min=1.0):
+    """T4 scale A: sum |terms| for I; for Q/U (k = 1, 2) at least eta_min * A_I, i.e. the
+    polarisation AMPLITUDE |eta cal| times sum |det_scale tod| (reading T4) — the
+    projected |Q| can vanish while the T2-allowed weight error does not."""
+    a = absmap.copy()
+    if a.shape[-1] == 3:
+        a[..., 1] = np.maximum(a[..., 1], eta_min * absmap[..., 0])
+        a[..., 2] = np.maximum(a[..., 2], eta_min * absmap[..., 0])
+    return a
+
+
+def check_map(gpu_map, ora_map, absmap, eta_min=0.98):
+    """T4 (scale from map_scale)."""
+    zero = absmap[..., :1] == 0 if absmap.shape[-1] == 3 else absmap == 0
+    zero = np.broadcast_to(zero, absmap.shape)
     assert np.all(gpu_map[zero] == 0.0), "map element with no contribution is not exactly 0"
     diff = np.abs(gpu_map - ora_map)
-    tol = 1e-10 * absmap
+    tol = 1e-10 * map_scale(absmap, eta_min)
     bad = diff > tol
     assert not np.any(bad), f"{int(bad.sum())} map elements beyond 1e-10 A; worst excess {(diff - tol).max()}"
 
