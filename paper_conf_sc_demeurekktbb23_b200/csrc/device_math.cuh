@@ -39,6 +39,7 @@ static __constant__ double kAtanQ[11] = {
 };
 
 constexpr double kTanPi8 = 0.41421356237309504880;
+static __constant__ double kHalfTurns[9] = {0.0, 0.5, 1.0, 1.5, 2.0, 2.5, 3.0, 3.5, 4.0};  // k / 2
 
 // 1/x for finite x > 0 (no IEEE rounding guarantee; <= ~1 ulp): MUFU seed + 2 Newton steps.
 __device__ __forceinline__ double fast_rcp(double x) {
@@ -95,15 +96,21 @@ __device__ __forceinline__ double small_int_to_double(int k) {
 
 __device__ __forceinline__ double qt_finish(const QtPrep& q, double t) {
     const double s = t * t;
-    // Estrin's scheme: dependency depth 5 instead of Horner's 10 (the kernel is latency-bound)
-    const double s2 = s * s, s4 = s2 * s2, s8 = s4 * s4;
-    const double q0 = fma(kAtanQ[1], s, kAtanQ[0]), q1 = fma(kAtanQ[3], s, kAtanQ[2]);
-    const double q2 = fma(kAtanQ[5], s, kAtanQ[4]), q3 = fma(kAtanQ[7], s, kAtanQ[6]);
-    const double q4 = fma(kAtanQ[9], s, kAtanQ[8]);
-    const double r0 = fma(q1, s2, q0), r1 = fma(q3, s2, q2), r2 = fma(kAtanQ[10], s2, q4);
-    const double p = fma(r2, s8, fma(r1, s4, r0));
+    // even/odd split Horner: depth 6 instead of 10, and every fma has ONE constant operand
+    // (a direct constant-bank operand, no extra constant loads; the kernel is issue-bound)
+    const double s2 = s * s;
+    double e = fma(kAtanQ[10], s2, kAtanQ[8]);
+    double o = fma(kAtanQ[9], s2, kAtanQ[7]);
+    e = fma(e, s2, kAtanQ[6]);
+    o = fma(o, s2, kAtanQ[5]);
+    e = fma(e, s2, kAtanQ[4]);
+    o = fma(o, s2, kAtanQ[3]);
+    e = fma(e, s2, kAtanQ[2]);
+    o = fma(o, s2, kAtanQ[1]);
+    e = fma(e, s2, kAtanQ[0]);
+    const double p = fma(o, s, e);
     const double tau = t * p;
-    double tt = fma(q.neg ? -1.0 : 1.0, tau, 0.5 * small_int_to_double(q.kk));
+    double tt = fma(q.neg ? -1.0 : 1.0, tau, kHalfTurns[q.kk]);
     if (tt >= 4.0) tt = 0.0;
     return tt;
 }
@@ -113,14 +120,31 @@ __device__ __forceinline__ double quarter_turns(double x, double y) {
     return qt_finish(q, q.num * fast_rcp(q.den));
 }
 
-// floor(x) for 0 <= x < 2^31 on the FP64 pipe (no F2I): rint via the 1.5 * 2^52 magic
-// number (the addition is exact up to the final rounding to an integer), then corrected by
-// one comparison — exact for every double in range, ties included.
+// floor(x) for 0 <= x < 2^31.  Default: one F2I (truncation = floor for x >= 0).  With
+// TB_FLOOR_FP64 it runs on the FP64 pipe instead: rint via the 1.5 * 2^52 magic number (the
+// addition is exact up to the final rounding to an integer), then corrected by one comparison
+// — exact for every double in range, ties included.  (Measured on B200: F2I is ~3% faster.)
 __device__ __forceinline__ int floor_nonneg(double x) {
+#ifndef TB_FLOOR_FP64
+    return (int)x;
+#else
     const double big = x + 6755399441055744.0;
     const double r = big - 6755399441055744.0;  // rint(x), exact
     const int n = __double2loint(big);
     return (r > x) ? n - 1 : n;
+#endif
+}
+
+// sqrt(x) for x >= 0.03 (the HEALPix cap term 3(1 - |z|) with |z| < 0.99): reciprocal square
+// root seed + two Newton steps, within ~1 ulp (not IEEE-rounded; only floors of it matter, and
+// those may differ from the oracle only within ~1e-15 rad of a pixel boundary).
+__device__ __forceinline__ double fast_sqrt(double x) {
+    double y;
+    asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(x));
+    y = y * fma(-0.5 * x, y * y, 1.5);
+    y = y * fma(-0.5 * x, y * y, 1.5);
+    const double r = x * y;
+    return fma(0.5 * y, fma(-r, r, x), r);  // one Newton step on sqrt itself
 }
 
 // sin and cos of a moderate angle (|a| < 2^20 pi/2; here a = 4 chi in [0, 8 pi)): Cody-Waite
@@ -330,7 +354,7 @@ __device__ __forceinline__ int loc2pix32(const HealpixGeom& g, double dz, double
     }
     double tmp;
     if (za < 0.99) {
-        tmp = __dmul_rn(g.dnside, __dsqrt_rn(__dmul_rn(3.0, __dsub_rn(1.0, za))));
+        tmp = __dmul_rn(g.dnside, fast_sqrt(__dmul_rn(3.0, __dsub_rn(1.0, za))));
     } else {
         const double sth = __dsqrt_rn(__dadd_rn(__dmul_rn(dx, dx), __dmul_rn(dy, dy)));
         tmp = __ddiv_rn(__dmul_rn(g.dnside, sth), __dsqrt_rn(__ddiv_rn(__dadd_rn(1.0, za), 3.0)));

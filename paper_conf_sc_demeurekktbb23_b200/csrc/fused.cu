@@ -463,12 +463,25 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
             sm.st[lane] = x;
         }
         const unsigned pmask = __ballot_sync(0xffffffffu, pixelise_me);
-        int foff[DPL];
+        // det flags of the lane's rows -> one bit per sample (bit k: sample k is det-flagged)
+        unsigned fmask[DPL];
 #pragma unroll
-        for (int j = 0; j < DPL; ++j)
-            foff[j] = have_dflags
-                          ? (int)(reinterpret_cast<uintptr_t>(a.det_flags + (cur.d0 + lane + 32 * j) * a.n_samp + cur.s0) & 3)
-                          : 0;
+        for (int j = 0; j < DPL; ++j) {
+            fmask[j] = 0u;
+            const int row = lane + 32 * j;
+            if (have_dflags && row < cur.nrows) {
+                const int foff =
+                    (int)(reinterpret_cast<uintptr_t>(a.det_flags + (cur.d0 + row) * a.n_samp + cur.s0) & 3);
+                const unsigned rep = dmask * 0x01010101u;
+                unsigned bits = 0u;  // bit b: byte b of the 20-byte window is flagged
+#pragma unroll
+                for (int w = 0; w < 5; ++w) {
+                    const unsigned v = __vcmpne4(*reinterpret_cast<const unsigned*>(&rb.flg[row][4 * w]) & rep, 0u);
+                    bits |= ((v & 0x01010101u) * 0x01020408u >> 24 & 0xfu) << (4 * w);
+                }
+                fmask[j] = (bits >> foff) & ((cur.nb >= 32) ? 0xffffffffu : ((1u << cur.nb) - 1u));
+            }
+        }
         __syncwarp();
 
 #pragma unroll 1
@@ -488,7 +501,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
             for (int j = 0; j < DPL; ++j) {
                 const int row = lane + 32 * j;
                 tod[j] = rb.tod[row][k];
-                dflag[j] = have_dflags && ((rb.flg[row][k + foff[j]] & dmask) != 0);
+                dflag[j] = (fmask[j] >> k) & 1u;
             }
             // fold the previous sample while those shared-memory loads are in flight
 #pragma unroll
