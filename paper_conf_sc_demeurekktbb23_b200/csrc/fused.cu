@@ -251,56 +251,8 @@ __device__ __forceinline__ void det_sample(Slot<typename PixT<WIDE>::T>& sl, con
 
 // Fold the pending contribution into the run (run-length aggregation along time).  Lanes
 // without a pixel (no detector / flagged sample) have pend_pix = -1 and never touch their run.
-__device__ __forceinline__ void red_if(bool p, double* addr, double v) {
-    asm volatile("{\n .reg .pred q;\n setp.ne.u32 q, %0, 0;\n @q red.global.add.f64 [%1], %2;\n}\n" ::"r"((unsigned)p),
-                 "l"(addr), "d"(v)
-                 : "memory");
-}
-__device__ __forceinline__ int64_t ldg_if(bool p, const int64_t* addr, int64_t dflt) {
-    int64_t v = dflt;
-    asm volatile("{\n .reg .pred q;\n setp.ne.u32 q, %1, 0;\n @q ld.global.nc.s64 %0, [%2];\n}\n"
-                 : "+l"(v)
-                 : "r"((unsigned)p), "l"(addr));
-    return v;
-}
-__device__ __forceinline__ void stg_u8_if(bool p, uint8_t* addr) {
-    asm volatile("{\n .reg .pred q;\n setp.ne.u32 q, %0, 0;\n @q st.global.u8 [%1], 1;\n}\n" ::"r"((unsigned)p),
-                 "l"(addr)
-                 : "memory");
-}
-
 template <int NNZ, typename P>
 __device__ __forceinline__ void aggregate(Slot<P>& sl, const FusedArgs& a) {
-#ifdef TB_BRANCHFREE_AGG
-    // branch-free form: predicated red / ld / st, so a rare run end in one lane does not
-    // make the whole warp take a divergent path
-    const MapGeom& mg = a.map;
-    const bool has = sl.pend_pix >= 0;
-    const bool newrun = has && sl.pend_pix != sl.run_pix;
-    const bool doflush = newrun && sl.run_pix >= 0 && sl.run_loc >= 0;
-    const P fp = sl.run_pix < 0 ? 0 : sl.run_pix;
-    const int64_t lp = mg.sm_shift >= 0 ? (int64_t)(fp & (P)(mg.n_pix_submap - 1))
-                                        : (int64_t)fp - submap_of<P>(fp, mg) * mg.n_pix_submap;
-    double* dst = a.zmap + (sl.run_loc * mg.n_pix_submap + lp) * NNZ;
-    red_if(doflush, dst, sl.r0);
-    if (NNZ == 3) {
-        red_if(doflush, dst + 1, sl.r1);
-        red_if(doflush, dst + 2, sl.r2);
-    }
-    const P np = has ? sl.pend_pix : 0;
-    const int64_t sm = submap_of<P>(np, mg);
-    if (a.hit_submaps) stg_u8_if(newrun, a.hit_submaps + sm);
-    sl.run_loc = ldg_if(newrun, mg.global2local + sm, sl.run_loc);
-    sl.run_pix = newrun ? sl.pend_pix : sl.run_pix;
-    sl.r0 = (newrun ? 0.0 : sl.r0) + (has ? sl.p0 : 0.0);
-    if (NNZ == 3) {
-        sl.r1 = (newrun ? 0.0 : sl.r1) + (has ? sl.p1 : 0.0);
-        sl.r2 = (newrun ? 0.0 : sl.r2) + (has ? sl.p2 : 0.0);
-    }
-    sl.pend_pix = -1;
-    sl.p0 = sl.p1 = sl.p2 = 0.0;
-    return;
-#endif
     if (sl.pend_pix >= 0) {
         if (sl.pend_pix != sl.run_pix) {
 #ifndef TB_X_NOFLUSH
