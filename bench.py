@@ -57,6 +57,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--soak", type=float, default=1.0, help="seconds of untimed steps before timing (clocks)")
+    ap.add_argument("--reduce", default="auto", choices=["auto", "dense", "packed"],
+                    help="N>1 map reduction: dense all_reduce, or all_reduce of the union of hit submaps")
     return ap.parse_args()
 
 
@@ -219,6 +221,7 @@ def main():
     import torch
     import torch.distributed as dist
     from paper_conf_sc_demeurekktbb23_b200 import binding, synth
+    from paper_conf_sc_demeurekktbb23_b200 import dist as tdist
     from paper_conf_sc_demeurekktbb23_b200.staging import DeviceWorkload
 
     if not torch.cuda.is_available():
@@ -236,8 +239,13 @@ def main():
     lib = binding.load()
     call = lib.toast_pointing_to_map
 
+    packed = args.reduce == "packed" or (args.reduce == "auto" and dw.zmap.numel() * 8 > (256 << 20))
+    reduced = [0]
+
     def step(k0=None, k1=None):
         dw.zmap.zero_()
+        if packed:
+            dw.hit_submaps.zero_()
         if k0 is not None:
             k0.record(stream)
         rc = call(*raw)
@@ -246,7 +254,11 @@ def main():
         if k1 is not None:
             k1.record(stream)
         if world > 1:
-            dist.all_reduce(dw.zmap, op=dist.ReduceOp.SUM)
+            if packed:
+                tdist.union_hit_submaps(dw.hit_submaps)
+                _, reduced[0] = tdist.reduce_map(dw.zmap, hit_submaps=dw.hit_submaps, global2local=dw.global2local)
+            else:
+                _, reduced[0] = tdist.reduce_map(dw.zmap)
 
     for _ in range(max(3, args.warmup)):
         step()
@@ -329,7 +341,10 @@ def main():
                            "l2": f"inputs larger than L2 (TOD {w.det_data.nbytes / 1e6:.0f} MB per rank), no flush",
                            "parallelism": f"dp{world} (one observation per rank + NCCL all-reduce of the map)"
                            if world > 1 else "single GPU",
-                           "step": "zero map + toast_pointing_to_map" + (" + all_reduce(map)" if world > 1 else "")},
+                           "step": "zero map + toast_pointing_to_map" + (
+                               (" + all_reduce(hit submaps, MAX) + packed all_reduce(map)" if packed
+                                else " + all_reduce(map)") if world > 1 else ""),
+                           "allreduce_bytes_per_step": reduced[0]},
                 "clocks": clocks, "gpu_launches": args.steps, "roofline": roofline}
         if e2e is not None:
             line["e2e"] = e2e
