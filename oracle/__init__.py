@@ -78,6 +78,8 @@ def _declare(L):
                                              P, I64, I64, INT]
     L.oracle_pointing_to_map_omp.restype = INT
     L.oracle_det_sample_probe.argtypes = [P, P, D, D, D, INT, I64, INT, P, P, P]
+    L.oracle_pointing_to_tod.argtypes = [P, P, P, P, D, P, U8, P, I64, I64, INT, I64, P, I64, P, D, INT, INT, P, I64,
+                                         I64, P]
 
 
 def _p(a):
@@ -262,3 +264,19 @@ def pointing_to_map_omp(fp_quats, boresight, epsilon, cal, det_scale, det_data, 
         _p(_arr(det_scale, np.float64)), _p(_arr(det_data, np.float64)), _p(_arr(det_flags, np.uint8)),
         det_flag_mask, _p(_arr(shared_flags, np.uint8)), shared_flag_mask, _p(iv), len(iv), nside, int(nest), nnz,
         _p(_arr(global2local, np.int64)), n_pix_submap, _p(zmap), n_det, n_samp, int(n_threads)))
+
+
+def pointing_to_tod(fp_quats, boresight, epsilon, cal, intervals, nside, nest, nnz, global2local, n_pix_submap,
+                    mapdata, det_data, data_scale=1.0, should_zero=False, should_subtract=False, hwp=None,
+                    shared_flags=None, shared_flag_mask=0, bscale=None):
+    """f1: A1 -> A2 -> A3 -> A5 per det-sample (scan a map onto the timestream in place)."""
+    fp = _arr(fp_quats, np.float64); bore = _arr(boresight, np.float64)
+    n_det, n_samp = fp.shape[0], bore.shape[0]
+    iv = intervals_array(intervals) if not isinstance(intervals, np.ndarray) else intervals
+    assert det_data.dtype == np.float64 and det_data.flags["C_CONTIGUOUS"] and det_data.shape == (n_det, n_samp)
+    lib().oracle_pointing_to_tod(_p(fp), _p(bore), _p(_arr(hwp, np.float64)), _p(_arr(epsilon, np.float64)),
+                                 float(cal), _p(_arr(shared_flags, np.uint8)), shared_flag_mask, _p(iv), len(iv),
+                                 nside, int(nest), nnz, _p(_arr(global2local, np.int64)), n_pix_submap,
+                                 _p(_arr(mapdata, np.float64)), float(data_scale), int(should_zero),
+                                 int(should_subtract), _p(det_data), n_det, n_samp, _p(bscale))
+    return det_data

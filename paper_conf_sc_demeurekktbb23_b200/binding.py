@@ -54,15 +54,18 @@ def load():
     L.toast_scan_map.argtypes = [P, I64, P, I64, P, P, P, P, P, P, P, I64, D, I32, I32, I64, I64, P]
     L.toast_pointing_to_map.argtypes = [P, P, P, P, D, P, P, P, U8, P, U8, P, I64, I64, I32, I64, P, I64, P, P, P, P,
                                         I64, I64, P]
+    L.toast_pointing_to_tod.argtypes = [P, P, P, P, D, P, U8, P, I64, I64, I32, I64, P, I64, P, D, I32, I32, P, I64,
+                                        I64, P]
     for name in ("toast_pointing_detector", "toast_pixels_healpix", "toast_stokes_weights_iqu",
-                 "toast_build_noise_weighted", "toast_scan_map", "toast_pointing_to_map"):
+                 "toast_build_noise_weighted", "toast_scan_map", "toast_pointing_to_map", "toast_pointing_to_tod"):
         getattr(L, name).restype = I32
     _lib = L
     return L
 
 
 EXPORTED = ("toast_last_error", "toast_version", "toast_release", "toast_pointing_detector", "toast_pixels_healpix",
-            "toast_stokes_weights_iqu", "toast_build_noise_weighted", "toast_scan_map", "toast_pointing_to_map")
+            "toast_stokes_weights_iqu", "toast_build_noise_weighted", "toast_scan_map", "toast_pointing_to_map",
+            "toast_pointing_to_tod")
 
 
 def version() -> str:
@@ -210,6 +213,23 @@ def pointing_to_map(fp_quats, boresight, epsilon, cal, det_scale, det_data, inte
         _stream(stream))
     _check(rc, "toast_pointing_to_map")
     return zmap
+
+
+def pointing_to_tod(fp_quats, boresight, epsilon, cal, intervals, nside, nest, nnz, global2local, n_pix_submap,
+                    mapdata, det_data, data_scale=1.0, should_zero=False, should_subtract=False, hwp=None,
+                    shared_flags=None, shared_flag_mask=0, stream=None):
+    """f1: fused A1 -> A2 -> A3 -> A5, scanning `mapdata` into `det_data` in place."""
+    n_det, n_samp = fp_quats.shape[0], boresight.shape[0]
+    keep, ivp, niv = _iv(intervals)
+    rc = load().toast_pointing_to_tod(
+        _dev(fp_quats, torch.float64, "fp_quats"), _dev(boresight, torch.float64, "boresight"),
+        _dev(hwp, torch.float64, "hwp"), _dev(epsilon, torch.float64, "epsilon"), float(cal),
+        _dev(shared_flags, torch.uint8, "shared_flags"), shared_flag_mask, ivp, niv, nside, int(nest), nnz,
+        _dev(global2local, torch.int64, "global2local"), n_pix_submap, _dev(mapdata, torch.float64, "mapdata"),
+        float(data_scale), int(should_zero), int(should_subtract), _dev(det_data, torch.float64, "det_data"), n_det,
+        n_samp, _stream(stream))
+    _check(rc, "toast_pointing_to_tod")
+    return det_data
 
 
 def pointing_to_map_raw(args: tuple):

@@ -399,3 +399,58 @@ int toast_pointing_to_map(const double* fp_quats, const double* boresight, const
 }
 
 }  // extern "C"
+
+extern "C" int toast_pointing_to_tod(const double* fp_quats, const double* boresight, const double* hwp,
+                                     const double* epsilon, double cal, const uint8_t* shared_flags,
+                                     uint8_t shared_flag_mask, const toast_interval_t* intervals, int64_t n_intervals,
+                                     int64_t nside, int nest, int64_t nnz, const int64_t* global2local,
+                                     int64_t n_pix_submap, const double* mapdata, double data_scale, int should_zero,
+                                     int should_subtract, double* det_data, int64_t n_det, int64_t n_samp,
+                                     void* stream) {
+    using namespace toastb200;
+    REQUIRE_DIMS(n_det, n_samp);
+    int rc = check_nside(nside);
+    if (rc != TOAST_OK) return rc;
+    if (nest != 0 && nest != 1) return fail(TOAST_EINVAL, "nest = %d must be 0 (RING) or 1 (NESTED)", nest);
+    if (nnz != 1 && nnz != 3) return fail(TOAST_EINVAL, "nnz = %lld must be 1 or 3", (long long)nnz);
+    rc = check_submap(n_pix_submap, 12 * nside * nside);
+    if (rc != TOAST_OK) return rc;
+    if (n_det > 0 && n_intervals > 0) {
+        REQUIRE(fp_quats);
+        REQUIRE(boresight);
+        REQUIRE(epsilon);
+        REQUIRE(global2local);
+        REQUIRE(mapdata);
+        REQUIRE(det_data);
+    }
+    WorkList wl;
+    rc = get_worklist(intervals, n_intervals, n_samp, &wl, kFusedChunk);
+    if (rc != TOAST_OK) return rc;
+    FusedArgs a = {};
+    a.fp_quats = fp_quats;
+    a.boresight = boresight;
+    a.hwp = hwp;
+    a.epsilon = epsilon;
+    a.cal = cal;
+    a.det_scale = epsilon;  // unused by the scan; any valid [n_det] array
+    a.det_data = det_data;
+    a.shared_flags = shared_flags;
+    a.shared_flag_mask = shared_flag_mask;
+    a.nside = nside;
+    a.nest = nest;
+    a.nnz = (int)nnz;
+    a.map = make_map_geom(global2local, n_pix_submap);
+    a.n_det = n_det;
+    a.n_samp = n_samp;
+    a.mapdata = mapdata;
+    a.data_scale = data_scale;
+    a.should_zero = should_zero;
+    a.should_subtract = should_subtract;
+    a.tod_out = det_data;
+    int serr = 0;
+    unsigned long long* sched = sched_counter(&serr);
+    if (serr) return fail(TOAST_ENOMEM, "could not allocate the work-distribution counter");
+    cudaError_t e = launch_pointing_to_tod(wl, a, sched, (cudaStream_t)stream);
+    if (e != cudaSuccess) return cuda_fail(e, "pointing_to_tod launch");
+    return ok();
+}

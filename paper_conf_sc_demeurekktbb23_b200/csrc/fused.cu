@@ -44,7 +44,15 @@ namespace {
 #define TB_FUSED_DPL_MAX 1  // detectors per lane (2 when n_det > 32 and DPL_MAX = 2)
 #endif
 constexpr int kWarps = 8;  // warps per CTA
-constexpr int kBlk = 16;   // samples per block
+#ifndef TB_BLK
+#define TB_BLK 16
+#endif
+constexpr int kBlk = TB_BLK;  // samples per block (8 or 16)
+constexpr int kRowStep = 32 / kBlk;  // TOD rows staged per cp.async instruction
+#ifndef TB_KUNROLL
+#define TB_KUNROLL 1
+#endif
+constexpr int kKUnroll = TB_KUNROLL;  // unroll of the per-sample loop
 constexpr int kPad = kBlk + 1;
 
 // per-sample state: B[0..8], c4, s4, mode (as a double: 1 pixelise, 2 shared-flagged)
@@ -72,9 +80,21 @@ __device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
     const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
 }
+// L2 evict-first policy for the streamed-once inputs (TOD, det flags): they must not push
+// the map lines being accumulated out of L2 (the map's red operations miss otherwise).
+__device__ __forceinline__ uint64_t evict_first_policy() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;\n" : "=l"(pol));
+    return pol;
+}
 __device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
     const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
     asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async8_stream(void* smem, const void* gmem, uint64_t pol) {
+    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 8, %2;\n" ::"r"(s), "l"(gmem), "l"(pol)
+                 : "memory");
 }
 __device__ __forceinline__ void cp_async4(void* smem, const void* gmem) {
     const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
@@ -287,15 +307,16 @@ __device__ __forceinline__ void issue_block(RawBlock<DPL>& rb, const Blk& bk, co
     constexpr int kRows = 32 * DPL;
     const int64_t n_samp = a.n_samp;
     const int scol = lane & (kBlk - 1);
-    const int srow = lane >> 4;  // 0 or 1
+    const int srow = lane / kBlk;
     if (scol < bk.nb) {
         const double* src = a.det_data + (bk.d0 + srow) * n_samp + bk.s0 + scol;
-        const int64_t step = 2 * n_samp;
+        const int64_t step = kRowStep * n_samp;
+        const uint64_t pol = evict_first_policy();
         if (bk.nrows == kRows) {
 #pragma unroll 8
-            for (int r = srow; r < kRows; r += 2, src += step) cp_async8(&rb.tod[r][scol], src);
+            for (int r = srow; r < kRows; r += kRowStep, src += step) cp_async8_stream(&rb.tod[r][scol], src, pol);
         } else {
-            for (int r = srow; r < bk.nrows; r += 2, src += step) cp_async8(&rb.tod[r][scol], src);
+            for (int r = srow; r < bk.nrows; r += kRowStep, src += step) cp_async8_stream(&rb.tod[r][scol], src, pol);
         }
     }
     // boresight: 16 quaternions = 32 x 16 B, one per lane
@@ -436,7 +457,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
         }
         __syncwarp();
 
-#pragma unroll 1
+#pragma unroll kKUnroll
         for (int k = 0; k < cur.nb; ++k) {
             const bool pixelise = (pmask >> k) & 1u;
             if (!DEBUG && !pixelise) continue;  // shared-flagged sample: nothing to add (uniform)
@@ -526,7 +547,253 @@ cudaError_t dispatch_hwp(const WorkList& wl, const FusedArgs& a, unsigned long l
     return dispatch_debug<NEST, NNZ, false>(wl, a, sched, st);
 }
 
+// ============================================================================ scan direction
+// toast_pointing_to_tod: A1 -> A2 -> A3 -> A5 per det-sample in registers,
+// the map GATHERED into the timestream in place.  Same item / block stream and per-sample
+// state as pointing_to_map_kernel (lane = detector, cp.async double buffer); per lane the map
+// values of the current pixel are cached across the run (one gather per pixel change, the
+// submap's global2local cached across runs), and the TOD update of sample k is completed at
+// sample k+1 so the gather latency hides behind one sample of pointing work.  The block's
+// TOD tile is updated in shared memory and written back coalesced.
+template <bool NEST, int NNZ, bool HWP, bool WIDE>
+__global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_tod_kernel(const Chunk* __restrict__ chunks,
+                                                                         int64_t n_chunks, FusedArgs a,
+                                                                         HealpixGeom g,
+                                                                         unsigned long long* __restrict__ sched) {
+    using P = typename PixT<WIDE>::T;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int lane = threadIdx.x & 31;
+    const int wid = threadIdx.x >> 5;
+    WarpSmem<1>& sm = reinterpret_cast<WarpSmem<1>*>(smem_raw)[wid];
+    const int64_t n_groups = (a.n_det + 31) / 32;
+    const int64_t n_items = n_chunks * n_groups;
+    const unsigned smask = a.shared_flag_mask;
+    const bool have_sflags = a.shared_flags != nullptr;
+    const MapGeom& mg = a.map;
+    const double ds = a.data_scale;
+    const double sgn = a.should_subtract ? -1.0 : 1.0;
+    const double keep = a.should_zero ? 0.0 : 1.0;
+
+    int64_t pend_item = -1, pend_first = 0;
+    int pend_count = 0;
+    auto prefetch_item = [&]() {
+        if (lane == 0) {
+            const unsigned long long it = atomicAdd(sched, 1ull);
+            pend_item = it < (unsigned long long)n_items ? (int64_t)it : -1;
+            if (pend_item >= 0) {
+                const Chunk ch = chunks[pend_item / n_groups];
+                pend_first = ch.first;
+                pend_count = ch.count;
+            }
+        }
+    };
+    auto take_item = [&]() -> Blk {
+        Blk bk;
+        bk.item = __shfl_sync(0xffffffffu, pend_item, 0);
+        const int64_t first = __shfl_sync(0xffffffffu, pend_first, 0);
+        const int count = __shfl_sync(0xffffffffu, pend_count, 0);
+        if (bk.item < 0) {
+            bk.d0 = bk.s0 = bk.s_end = 0;
+            bk.nb = bk.nrows = 0;
+            return bk;
+        }
+        const int64_t c = bk.item / n_groups;
+        bk.d0 = (bk.item - c * n_groups) * 32;
+        bk.nrows = (a.n_det - bk.d0) < 32 ? (int)(a.n_det - bk.d0) : 32;
+        bk.s0 = first;
+        bk.s_end = first + count;
+        bk.nb = count < kBlk ? count : kBlk;
+        return bk;
+    };
+
+    prefetch_item();
+    Blk cur = take_item();
+    if (cur.item < 0) return;
+    prefetch_item();
+    issue_block<1>(sm.buf[0], cur, a, false, HWP && NNZ == 3, lane);
+    Slot<P> sl;
+    load_slot<P>(sl, a, cur.d0 + lane, lane < cur.nrows, cur.d0);
+    int p = 0;
+    // per-lane gather cache: map values of pixel cur_pix (loc < 0: no storage)
+    P cur_pix = -1;
+    int64_t cur_loc = -1, last_sm = -1, last_loc = -1;
+    double m0 = 0.0, m1 = 0.0, m2 = 0.0;
+
+    while (true) {
+        Blk nxt;
+        if (cur.s0 + kBlk < cur.s_end) {
+            nxt = cur;
+            nxt.s0 = cur.s0 + kBlk;
+            nxt.nb = (nxt.s_end - nxt.s0) < kBlk ? (int)(nxt.s_end - nxt.s0) : kBlk;
+        } else {
+            nxt = take_item();
+            if (nxt.item >= 0) prefetch_item();
+        }
+        cp_async_wait_all();
+        __syncwarp();
+        if (nxt.item >= 0) issue_block<1>(sm.buf[p ^ 1], nxt, a, false, HWP && NNZ == 3, lane);
+
+        RawBlock<1>& rb = sm.buf[p];
+        bool pixelise_me = false;
+        if (lane < kBlk) {
+            double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 1.0;
+            double c4 = 1.0, s4 = 0.0;
+            if (lane < cur.nb) {
+                const int soff = have_sflags ? (int)(reinterpret_cast<uintptr_t>(a.shared_flags + cur.s0) & 3) : 0;
+                const bool flagged = have_sflags && (rb.sflg[soff + lane] & smask);
+                pixelise_me = !flagged;
+                if (!flagged) {
+                    q0 = rb.bore[lane][0]; q1 = rb.bore[lane][1]; q2 = rb.bore[lane][2]; q3 = rb.bore[lane][3];
+                }
+                if (HWP && NNZ == 3) small_sincos(4.0 * rb.hwp[lane], &s4, &c4);
+            }
+            SampleState x;
+            quat_to_matrix(q0, q1, q2, q3, x.v);
+            x.v[9] = c4;
+            x.v[10] = s4;
+            x.v[11] = 0.0;
+            sm.st[lane] = x;
+        }
+        const unsigned pmask = __ballot_sync(0xffffffffu, pixelise_me);
+        __syncwarp();
+
+        int pend_k = -1;  // sample whose TOD update waits for its gathered map values
+        double pend_tod = 0.0, pend_c2 = 0.0, pend_s2 = 0.0;
+        auto finish = [&]() {
+            if (pend_k >= 0) {
+                double t = m0 * a.cal;
+                if (NNZ == 3) t += sl.etacal * (m1 * pend_c2 + m2 * pend_s2);
+                rb.tod[lane][pend_k] = fma(sgn * ds, t, keep * pend_tod);
+                pend_k = -1;
+            }
+        };
+#pragma unroll 1
+        for (int k = 0; k < cur.nb; ++k) {
+            if (!((pmask >> k) & 1u)) continue;  // shared-flagged sample: no pixel, untouched (uniform)
+            double x[12];
+#pragma unroll
+            for (int i = 0; i < ((HWP && NNZ == 3) ? 12 : 10); i += 2) {
+                const double2 t2 = *reinterpret_cast<const double2*>(&sm.st[k].v[i]);
+                x[i] = t2.x;
+                x[i + 1] = t2.y;
+            }
+            const double tod = rb.tod[lane][k];
+            const double dx = x[0] * sl.u0 + x[1] * sl.u1 + x[2] * sl.u2;
+            const double dy = x[3] * sl.u0 + x[4] * sl.u1 + x[5] * sl.u2;
+            const double dz = x[6] * sl.u0 + x[7] * sl.u1 + x[8] * sl.u2;
+            double c2 = 0.0, s2 = 0.0, tt;
+            if (NNZ == 3) {
+                const double bx = x[6] * sl.v0 + x[7] * sl.v1 + x[8] * sl.v2;
+                const double by = -(x[6] * sl.w0 + x[7] * sl.w1 + x[8] * sl.w2);
+                tt = lon_pol(dx, dy, bx, by, c2, s2);
+                if (HWP) {
+                    const double c4 = x[9], s4 = x[10];
+                    const double cq = c2 * c4 - s2 * s4;
+                    const double sq = s2 * c4 + c2 * s4;
+                    c2 = cq;
+                    s2 = sq;
+                }
+            } else {
+                tt = quarter_turns(dx, dy);
+            }
+            P pix;
+            if (WIDE)
+                pix = (P)loc2pix<NEST, int64_t>(g, dz, tt, dx, dy);
+            else
+                pix = (P)loc2pix32<NEST>(g, dz, tt, dx, dy);
+            if (!sl.ok) pix = -1;
+            finish();  // the previous sample's gathered values have arrived by now
+            if (pix >= 0 && pix != cur_pix) {
+                const int64_t smi = submap_of<P>(pix, mg);
+                if (smi != last_sm) {
+                    last_loc = __ldg(&mg.global2local[smi]);
+                    last_sm = smi;
+                }
+                cur_pix = pix;
+                cur_loc = last_loc;
+                if (cur_loc >= 0) {
+                    const int64_t lp = mg.sm_shift >= 0 ? (int64_t)(pix & (P)(mg.n_pix_submap - 1))
+                                                        : (int64_t)pix - smi * mg.n_pix_submap;
+                    const double* mp = a.mapdata + (cur_loc * mg.n_pix_submap + lp) * NNZ;
+                    m0 = __ldg(mp);
+                    if (NNZ == 3) {
+                        m1 = __ldg(mp + 1);
+                        m2 = __ldg(mp + 2);
+                    }
+                }
+            }
+            if (pix >= 0 && cur_loc >= 0) {
+                pend_k = k;
+                pend_tod = tod;
+                pend_c2 = c2;
+                pend_s2 = s2;
+            }
+        }
+        finish();
+        __syncwarp();
+        // write the updated tile back (samples without a pixel keep the value read)
+        {
+            const int scol = lane & (kBlk - 1);
+            const int srow = lane / kBlk;
+            if (scol < cur.nb) {
+                double* dst = a.tod_out + (cur.d0 + srow) * a.n_samp + cur.s0 + scol;
+                const int64_t step = kRowStep * a.n_samp;
+                for (int r = srow; r < cur.nrows; r += kRowStep, dst += step) *dst = rb.tod[r][scol];
+            }
+        }
+        if (nxt.item != cur.item) {
+            if (nxt.item < 0) break;
+            load_slot<P>(sl, a, nxt.d0 + lane, lane < nxt.nrows, nxt.d0);
+            cur_pix = -1;
+            cur_loc = -1;
+        }
+        __syncwarp();
+        cur = nxt;
+        p ^= 1;
+    }
+    cp_async_wait_all();
+}
+
+template <bool NEST, int NNZ, bool HWP, bool WIDE>
+cudaError_t launch_scan_t(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
+    auto kern = pointing_to_tod_kernel<NEST, NNZ, HWP, WIDE>;
+    const size_t smem = sizeof(WarpSmem<1>) * kWarps;
+    static int blocks_per_sm = 0;
+    static std::once_flag once;
+    std::call_once(once, [&] {
+        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, kern, kWarps * 32, smem) != cudaSuccess ||
+            blocks_per_sm < 1)
+            blocks_per_sm = 1;
+    });
+    const int64_t n_items = wl.n_chunks * ((a.n_det + 31) / 32);
+    const int64_t want = (n_items + kWarps - 1) / kWarps;
+    const int64_t grid = std::min<int64_t>(want, (int64_t)num_sms() * blocks_per_sm);
+    if (grid <= 0) return cudaSuccess;
+    cudaError_t e = cudaMemsetAsync(sched, 0, sizeof(unsigned long long), st);
+    if (e != cudaSuccess) return e;
+    kern<<<(unsigned)grid, kWarps * 32, smem, st>>>(wl.chunks, wl.n_chunks, a, make_geom(a.nside), sched);
+    return cudaGetLastError();
+}
+
+template <bool NEST, int NNZ>
+cudaError_t dispatch_scan(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
+    const bool wide = a.nside > 8192;
+    const bool hwp = a.hwp && NNZ == 3;
+    if (wide) return hwp ? launch_scan_t<NEST, NNZ, true, true>(wl, a, sched, st)
+                         : launch_scan_t<NEST, NNZ, false, true>(wl, a, sched, st);
+    return hwp ? launch_scan_t<NEST, NNZ, true, false>(wl, a, sched, st)
+               : launch_scan_t<NEST, NNZ, false, false>(wl, a, sched, st);
+}
+
 }  // namespace
+
+cudaError_t launch_pointing_to_tod(const WorkList& wl, const FusedArgs& a, unsigned long long* sched,
+                                   cudaStream_t st) {
+    if (wl.n_chunks == 0 || a.n_det == 0) return cudaSuccess;
+    if (a.nest) return a.nnz == 3 ? dispatch_scan<true, 3>(wl, a, sched, st) : dispatch_scan<true, 1>(wl, a, sched, st);
+    return a.nnz == 3 ? dispatch_scan<false, 3>(wl, a, sched, st) : dispatch_scan<false, 1>(wl, a, sched, st);
+}
 
 cudaError_t launch_pointing_to_map(const WorkList& wl, const FusedArgs& a, unsigned long long* sched,
                                    cudaStream_t st) {

@@ -55,6 +55,12 @@ struct FusedArgs {
     double* weights_out;
     int64_t n_det;
     int64_t n_samp;
+    // pointing_to_tod (scan direction) only
+    const double* mapdata;
+    double data_scale;
+    int should_zero;
+    int should_subtract;
+    double* tod_out;
 };
 
 cudaError_t launch_pointing_detector(const WorkList& wl, const double* fp_quats, const double* boresight,
@@ -81,6 +87,8 @@ cudaError_t launch_scan_map(const WorkList& wl, const MapGeom& mg, const double*
                             double data_scale, int should_zero, int should_subtract, int64_t n_det, int64_t n_samp,
                             cudaStream_t st);
 cudaError_t launch_pointing_to_map(const WorkList& wl, const FusedArgs& a, unsigned long long* sched,
+                                   cudaStream_t st);
+cudaError_t launch_pointing_to_tod(const WorkList& wl, const FusedArgs& a, unsigned long long* sched,
                                    cudaStream_t st);
 
 // A device counter for dynamic work distribution (zeroed on the stream before each use).

@@ -199,3 +199,51 @@ def test_omp_mode_matches_sequential(small):
                                       shared_flags=w.shared_flags, shared_flag_mask=w.shared_flag_mask, n_threads=2)
     assert used >= 1
     np.testing.assert_allclose(z2, z1, rtol=1e-12, atol=1e-12)
+
+
+def test_pointing_to_tod_equals_composition_and_modes(small):
+    """f1 pointing_to_tod == A1 -> A2 -> A3 -> A5 (oracle entries), for each tod mode."""
+    w = small
+    quats = oracle.pointing_detector(w.fp_quats, w.boresight, w.intervals, w.shared_flags, w.shared_flag_mask)
+    pix, _ = oracle.pixels_healpix(quats, w.intervals, w.nside, w.nest, w.n_pix_submap, w.shared_flags,
+                                   w.shared_flag_mask)
+    wts = oracle.stokes_weights_iqu(quats, w.intervals, w.epsilon, w.cal, hwp=w.hwp)
+    rng = np.random.default_rng(71)
+    m = rng.normal(size=(w.n_submap, w.n_pix_submap, 3))
+    for zero, sub in ((False, False), (True, False), (False, True)):
+        t1 = w.det_data.copy()
+        oracle.scan_map(m, w.global2local, w.n_pix_submap, pix, wts, t1, w.intervals, data_scale=0.3,
+                        should_zero=zero, should_subtract=sub)
+        t2 = w.det_data.copy()
+        oracle.pointing_to_tod(w.fp_quats, w.boresight, w.epsilon, w.cal, w.intervals, w.nside, w.nest, 3,
+                               w.global2local, w.n_pix_submap, m, t2, data_scale=0.3, should_zero=zero,
+                               should_subtract=sub, hwp=w.hwp, shared_flags=w.shared_flags,
+                               shared_flag_mask=w.shared_flag_mask)
+        np.testing.assert_array_equal(t2, t1)
+
+
+def test_pointing_to_tod_constant_map_and_adjoint(small):
+    """Constant I map scans to data_scale * c * cal exactly; <scan(m), t> = <m, accumulate(t)>
+    with det_scale = 1 and no det flags."""
+    w = small
+    m = np.zeros((w.n_submap, w.n_pix_submap, 3)); m[..., 0] = 1.75
+    tod = np.full((w.n_det, w.n_samp), 9.0)
+    oracle.pointing_to_tod(w.fp_quats, w.boresight, w.epsilon, w.cal, w.intervals, w.nside, w.nest, 3,
+                           w.global2local, w.n_pix_submap, m, tod, data_scale=2.0, should_zero=True, hwp=w.hwp,
+                           shared_flags=w.shared_flags, shared_flag_mask=w.shared_flag_mask)
+    inside = _mask_intervals(w.intervals, w.n_samp) & ((w.shared_flags & w.shared_flag_mask) == 0)
+    assert np.all(tod[:, inside] == 2.0 * 1.75 * w.cal)
+    assert np.all(tod[:, ~inside] == 9.0)
+    rng = np.random.default_rng(72)
+    m = rng.normal(size=(w.n_submap, w.n_pix_submap, 3))
+    t = rng.normal(size=(w.n_det, w.n_samp))
+    scanned = np.zeros((w.n_det, w.n_samp))
+    oracle.pointing_to_tod(w.fp_quats, w.boresight, w.epsilon, w.cal, w.intervals, w.nside, w.nest, 3,
+                           w.global2local, w.n_pix_submap, m, scanned, hwp=w.hwp, shared_flags=w.shared_flags,
+                           shared_flag_mask=w.shared_flag_mask)
+    z = np.zeros_like(m)
+    oracle.pointing_to_map(w.fp_quats, w.boresight, w.epsilon, w.cal, np.ones(w.n_det), t, w.intervals, w.nside,
+                           w.nest, 3, w.global2local, w.n_pix_submap, zmap=z, hwp=w.hwp, shared_flags=w.shared_flags,
+                           shared_flag_mask=w.shared_flag_mask)
+    lhs, rhs = float(np.sum(scanned * t)), float(np.sum(z * m))
+    assert abs(lhs - rhs) <= 1e-12 * (float(np.sum(np.abs(scanned * t))) + 1.0)

@@ -399,3 +399,50 @@ def test_invalid_arguments_are_rejected():
     with pytest.raises(binding.ToastError, match="CUDA tensor"):
         binding.pointing_to_map(dw.fp_quats.cpu(), dw.boresight, dw.epsilon, 1.0, dw.det_scale, dw.det_data,
                                 w.intervals, w.nside, False, 3, dw.global2local, w.n_pix_submap, dw.zmap)
+
+
+# ----------------------------------------------------------------------------- f1 pointing_to_tod
+
+SCAN_CASES = {
+    "c1_ring": dict(name="c1", n_samp=60_000),
+    "c2_nest_hwp_flags": dict(name="c2", n_det=40, n_samp=120_000),
+    "c2_nnz1": dict(name="c2", n_det=12, n_samp=60_000, nnz=1),
+    "c3_ring_flags": dict(name="c3", n_det=36, n_samp=30_000),
+    "c5_nest_4096": dict(name="c5", n_det=20, n_samp=60_000),
+}
+
+
+@pytest.mark.parametrize("case", list(SCAN_CASES))
+@pytest.mark.parametrize("mode", ["add", "zero", "subtract"])
+def test_fused_pointing_to_tod(case, mode):
+    w = synth.make_workload(**SCAN_CASES[case])
+    rng = np.random.default_rng(81)
+    m = rng.normal(size=(w.n_submap, w.n_pix_submap, w.nnz))
+    zero, sub = mode == "zero", mode == "subtract"
+    ref = w.det_data.copy()
+    b = np.zeros_like(ref)
+    oracle.pointing_to_tod(w.fp_quats, w.boresight, w.epsilon, w.cal, w.intervals, w.nside, w.nest, w.nnz,
+                           w.global2local, w.n_pix_submap, m, ref, data_scale=0.8, should_zero=zero,
+                           should_subtract=sub, hwp=w.hwp, shared_flags=w.shared_flags,
+                           shared_flag_mask=w.shared_flag_mask, bscale=b)
+    dw = DeviceWorkload.upload(w, DEV)
+    tg = dw.det_data.clone()
+    binding.pointing_to_tod(dw.fp_quats, dw.boresight, dw.epsilon, w.cal, w.intervals, w.nside, w.nest, w.nnz,
+                            dw.global2local, w.n_pix_submap, _cuda(m, torch.float64), tg, data_scale=0.8,
+                            should_zero=zero, should_subtract=sub, hwp=dw.hwp, shared_flags=dw.shared_flags,
+                            shared_flag_mask=w.shared_flag_mask)
+    got = tg.cpu().numpy()
+    # T3: 1e-12 of the scanned magnitude, plus the T2 weight tolerance carried by the map values
+    quats = oracle.pointing_detector(w.fp_quats, w.boresight, w.intervals, w.shared_flags, w.shared_flag_mask)
+    eta_cal = (1 - w.epsilon) / (1 + w.epsilon) * w.cal
+    wtol = np.abs(eta_cal)[:, None] * np.maximum(1e-12, 1e-15 / np.maximum(_sin_theta(quats), 1e-300))
+    mabs = float(np.abs(m).max())
+    tol = 1e-12 * b + 0.8 * mabs * 2 * wtol + 4e-16 * np.abs(ref) + 1e-300
+    bad = np.nonzero(np.abs(got - ref) > tol)
+    n_in = int(_in_mask(w.intervals, 1, w.n_samp).sum()) * w.n_det
+    probe = _probe(w)
+    for d, s in zip(*bad):
+        assert oracle.near_boundary(w.nside, w.nest, probe(int(d), int(s))), f"tod mismatch at det {d} sample {s}"
+    assert len(bad[0]) <= 1e-6 * n_in
+    out = ~np.array(_in_mask(w.intervals, w.n_det, w.n_samp))
+    np.testing.assert_array_equal(got[out], w.det_data[out])  # out-of-interval samples untouched
