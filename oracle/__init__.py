@@ -280,3 +280,73 @@ def pointing_to_tod(fp_quats, boresight, epsilon, cal, intervals, nside, nest, n
                                  _p(_arr(mapdata, np.float64)), float(data_scale), int(should_zero),
                                  int(should_subtract), _p(det_data), n_det, n_samp, _p(bscale))
     return det_data
+
+
+# ----------------------------------------------------------------------------- NEXT rows (f2, f4)
+
+def _declare_next(L):
+    L.oracle_stokes_weights_i.argtypes = [P, P, D, P, I64, I64, I64]
+    L.oracle_noise_weight.argtypes = [P, P, P, P, I64, I64, I64]
+    L.oracle_template_offset_add_to_signal.argtypes = [I64, P, P, P, P, P, I64, I64, I64]
+    L.oracle_template_offset_project_signal.argtypes = [I64, P, P, P, P, P, P, U8, P, I64, I64, I64]
+    L.oracle_template_offset_apply_diag_precond.argtypes = [P, P, P, I64]
+
+
+def _lib_next():
+    L = lib()
+    if not getattr(L, "_next_declared", False):
+        _declare_next(L)
+        L._next_declared = True
+    return L
+
+
+def stokes_weights_i(weights, cal, intervals, n_det, weight_index=None):
+    iv = intervals_array(intervals) if not isinstance(intervals, np.ndarray) else intervals
+    _lib_next().oracle_stokes_weights_i(_p(_arr(weight_index, np.int32)), _p(weights), float(cal), _p(iv), len(iv),
+                                        n_det, weights.shape[1])
+    return weights
+
+
+def noise_weight(det_data, det_weights, intervals, data_index=None, n_det=None):
+    iv = intervals_array(intervals) if not isinstance(intervals, np.ndarray) else intervals
+    dw = _arr(det_weights, np.float64)
+    n_det = dw.shape[0] if n_det is None else n_det
+    _lib_next().oracle_noise_weight(_p(_arr(data_index, np.int32)), _p(det_data), _p(dw), _p(iv), len(iv), n_det,
+                                    det_data.shape[1])
+    return det_data
+
+
+def offset_amplitude_counts(intervals, step_length):
+    """Amplitudes per detector under reading O1: sum over intervals of ceil(len / step)."""
+    return int(sum((l - f + 1 + step_length - 1) // step_length for f, l in intervals))
+
+
+def template_offset_add_to_signal(step_length, amp_offset, amplitudes, det_data, intervals, data_index=None,
+                                  n_det=None):
+    iv = intervals_array(intervals) if not isinstance(intervals, np.ndarray) else intervals
+    ao = _arr(amp_offset, np.int64)
+    n_det = ao.shape[0] if n_det is None else n_det
+    _lib_next().oracle_template_offset_add_to_signal(step_length, _p(ao), _p(_arr(amplitudes, np.float64)),
+                                                     _p(_arr(data_index, np.int32)), _p(det_data), _p(iv), len(iv),
+                                                     n_det, det_data.shape[1])
+    return det_data
+
+
+def template_offset_project_signal(step_length, amp_offset, amplitudes, det_data, intervals, det_flags=None,
+                                   det_flag_mask=0, data_index=None, flag_index=None, n_det=None):
+    iv = intervals_array(intervals) if not isinstance(intervals, np.ndarray) else intervals
+    ao = _arr(amp_offset, np.int64)
+    n_det = ao.shape[0] if n_det is None else n_det
+    dd = _arr(det_data, np.float64)
+    _lib_next().oracle_template_offset_project_signal(step_length, _p(ao), _p(amplitudes),
+                                                      _p(_arr(data_index, np.int32)), _p(dd),
+                                                      _p(_arr(flag_index, np.int32)), _p(_arr(det_flags, np.uint8)),
+                                                      det_flag_mask, _p(iv), len(iv), n_det, dd.shape[1])
+    return amplitudes
+
+
+def template_offset_apply_diag_precond(offset_var, amp_in):
+    ov = _arr(offset_var, np.float64); ai = _arr(amp_in, np.float64)
+    out = np.zeros_like(ai)
+    _lib_next().oracle_template_offset_apply_diag_precond(_p(ov), _p(ai), _p(out), ai.shape[0])
+    return out

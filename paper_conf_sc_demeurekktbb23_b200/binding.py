@@ -56,8 +56,15 @@ def load():
                                         I64, I64, P]
     L.toast_pointing_to_tod.argtypes = [P, P, P, P, D, P, U8, P, I64, I64, I32, I64, P, I64, P, D, I32, I32, P, I64,
                                         I64, P]
+    L.toast_stokes_weights_i.argtypes = [P, P, D, P, I64, I64, I64, P]
+    L.toast_noise_weight.argtypes = [P, P, P, P, I64, I64, I64, P]
+    L.toast_template_offset_add_to_signal.argtypes = [I64, P, P, P, P, P, I64, I64, I64, P]
+    L.toast_template_offset_project_signal.argtypes = [I64, P, P, P, P, P, P, U8, P, I64, I64, I64, P]
+    L.toast_template_offset_apply_diag_precond.argtypes = [P, P, P, I64, P]
     for name in ("toast_pointing_detector", "toast_pixels_healpix", "toast_stokes_weights_iqu",
-                 "toast_build_noise_weighted", "toast_scan_map", "toast_pointing_to_map", "toast_pointing_to_tod"):
+                 "toast_build_noise_weighted", "toast_scan_map", "toast_pointing_to_map", "toast_pointing_to_tod",
+                 "toast_stokes_weights_i", "toast_noise_weight", "toast_template_offset_add_to_signal",
+                 "toast_template_offset_project_signal", "toast_template_offset_apply_diag_precond"):
         getattr(L, name).restype = I32
     _lib = L
     return L
@@ -65,7 +72,9 @@ def load():
 
 EXPORTED = ("toast_last_error", "toast_version", "toast_release", "toast_pointing_detector", "toast_pixels_healpix",
             "toast_stokes_weights_iqu", "toast_build_noise_weighted", "toast_scan_map", "toast_pointing_to_map",
-            "toast_pointing_to_tod")
+            "toast_pointing_to_tod", "toast_stokes_weights_i", "toast_noise_weight",
+            "toast_template_offset_add_to_signal", "toast_template_offset_project_signal",
+            "toast_template_offset_apply_diag_precond")
 
 
 def version() -> str:
@@ -230,6 +239,56 @@ def pointing_to_tod(fp_quats, boresight, epsilon, cal, intervals, nside, nest, n
         n_samp, _stream(stream))
     _check(rc, "toast_pointing_to_tod")
     return det_data
+
+
+def stokes_weights_i(weights, cal, intervals, n_det=None, weight_index=None, stream=None):
+    n_det = weights.shape[0] if n_det is None else n_det
+    keep, ivp, niv = _iv(intervals)
+    _check(load().toast_stokes_weights_i(_dev(weight_index, torch.int32, "weight_index"),
+                                         _dev(weights, torch.float64, "weights"), float(cal), ivp, niv, n_det,
+                                         weights.shape[1], _stream(stream)), "toast_stokes_weights_i")
+    return weights
+
+
+def noise_weight(det_data, det_weights, intervals, data_index=None, n_det=None, stream=None):
+    n_det = det_weights.shape[0] if n_det is None else n_det
+    keep, ivp, niv = _iv(intervals)
+    _check(load().toast_noise_weight(_dev(data_index, torch.int32, "data_index"),
+                                     _dev(det_data, torch.float64, "det_data"),
+                                     _dev(det_weights, torch.float64, "det_weights"), ivp, niv, n_det,
+                                     det_data.shape[1], _stream(stream)), "toast_noise_weight")
+    return det_data
+
+
+def template_offset_add_to_signal(step_length, amp_offset, amplitudes, det_data, intervals, data_index=None,
+                                  n_det=None, stream=None):
+    n_det = amp_offset.shape[0] if n_det is None else n_det
+    keep, ivp, niv = _iv(intervals)
+    _check(load().toast_template_offset_add_to_signal(
+        int(step_length), _dev(amp_offset, torch.int64, "amp_offset"), _dev(amplitudes, torch.float64, "amplitudes"),
+        _dev(data_index, torch.int32, "data_index"), _dev(det_data, torch.float64, "det_data"), ivp, niv, n_det,
+        det_data.shape[1], _stream(stream)), "toast_template_offset_add_to_signal")
+    return det_data
+
+
+def template_offset_project_signal(step_length, amp_offset, amplitudes, det_data, intervals, det_flags=None,
+                                   det_flag_mask=0, data_index=None, flag_index=None, n_det=None, stream=None):
+    n_det = amp_offset.shape[0] if n_det is None else n_det
+    keep, ivp, niv = _iv(intervals)
+    _check(load().toast_template_offset_project_signal(
+        int(step_length), _dev(amp_offset, torch.int64, "amp_offset"), _dev(amplitudes, torch.float64, "amplitudes"),
+        _dev(data_index, torch.int32, "data_index"), _dev(det_data, torch.float64, "det_data"),
+        _dev(flag_index, torch.int32, "flag_index"), _dev(det_flags, torch.uint8, "det_flags"), det_flag_mask, ivp,
+        niv, n_det, det_data.shape[1], _stream(stream)), "toast_template_offset_project_signal")
+    return amplitudes
+
+
+def template_offset_apply_diag_precond(offset_var, amp_in, amp_out, stream=None):
+    _check(load().toast_template_offset_apply_diag_precond(
+        _dev(offset_var, torch.float64, "offset_var"), _dev(amp_in, torch.float64, "amp_in"),
+        _dev(amp_out, torch.float64, "amp_out"), amp_in.numel(), _stream(stream)),
+        "toast_template_offset_apply_diag_precond")
+    return amp_out
 
 
 def pointing_to_map_raw(args: tuple):

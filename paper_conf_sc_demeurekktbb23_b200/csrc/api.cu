@@ -187,6 +187,8 @@ unsigned long long* sched_counter(int* err) {
     return pools[dev] + (next[dev]++ % kPool) * (128 / sizeof(unsigned long long));
 }
 
+void release_offset_cache();
+
 int num_sms() {
     static int sms[64] = {0};
     int dev = 0;
@@ -220,6 +222,7 @@ int toast_release(void) {
     }
     cudaSetDevice(cur);
     g_cache.clear();
+    release_offset_cache();
     return ok();
 }
 
@@ -452,5 +455,172 @@ extern "C" int toast_pointing_to_tod(const double* fp_quats, const double* bores
     if (serr) return fail(TOAST_ENOMEM, "could not allocate the work-distribution counter");
     cudaError_t e = launch_pointing_to_tod(wl, a, sched, (cudaStream_t)stream);
     if (e != cudaSuccess) return cuda_fail(e, "pointing_to_tod launch");
+    return ok();
+}
+
+// ---------------------------------------------------------------- NEXT rows (f2, f4)
+
+namespace toastb200 {
+namespace {
+
+struct OffsetCacheEntry {
+    int device;
+    int step;
+    std::vector<toast_interval_t> intervals;
+    int64_t* d_arrays;  // [2][n]: iv_first, view_base
+};
+std::mutex g_ocache_mu;
+std::vector<OffsetCacheEntry> g_ocache;
+
+int get_offset_views(const toast_interval_t* iv, int64_t n, int64_t step, OffsetViews* out) {
+    if (step < 1 || step > (int64_t(1) << 30)) return fail(TOAST_EINVAL, "step_length = %lld must be in [1, 2^30]",
+                                                           (long long)step);
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    std::lock_guard<std::mutex> lk(g_ocache_mu);
+    for (auto& c : g_ocache) {
+        if (c.device == dev && c.step == (int)step && (int64_t)c.intervals.size() == n &&
+            (n == 0 || std::memcmp(c.intervals.data(), iv, sizeof(toast_interval_t) * n) == 0)) {
+            *out = OffsetViews{c.d_arrays, c.d_arrays + n, (int)step};
+            return TOAST_OK;
+        }
+    }
+    std::vector<int64_t> h(2 * std::max<int64_t>(n, 1), 0);
+    int64_t base = 0;
+    for (int64_t i = 0; i < n; ++i) {
+        h[i] = iv[i].first;
+        h[n + i] = base;
+        const int64_t len = iv[i].last - iv[i].first + 1;
+        base += (len + step - 1) / step;
+    }
+    int64_t* d = nullptr;
+    e = cudaMalloc(&d, sizeof(int64_t) * h.size());
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(TOAST_ENOMEM, "cudaMalloc of the offset views: %s", cudaGetErrorString(e));
+    }
+    e = cudaMemcpy(d, h.data(), sizeof(int64_t) * h.size(), cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) {
+        cudaFree(d);
+        return cuda_fail(e, "cudaMemcpy of the offset views");
+    }
+    if (g_ocache.size() >= kCacheMax) {
+        int cur = dev;
+        cudaSetDevice(g_ocache.front().device);
+        cudaFree(g_ocache.front().d_arrays);
+        cudaSetDevice(cur);
+        g_ocache.erase(g_ocache.begin());
+    }
+    g_ocache.push_back(OffsetCacheEntry{dev, (int)step, std::vector<toast_interval_t>(iv, iv + n), d});
+    *out = OffsetViews{d, d + n, (int)step};
+    return TOAST_OK;
+}
+
+}  // namespace
+
+void release_offset_cache() {
+    std::lock_guard<std::mutex> lk(g_ocache_mu);
+    int cur = 0;
+    cudaGetDevice(&cur);
+    for (auto& c : g_ocache) {
+        cudaSetDevice(c.device);
+        cudaFree(c.d_arrays);
+    }
+    cudaSetDevice(cur);
+    g_ocache.clear();
+}
+
+}  // namespace toastb200
+
+extern "C" int toast_stokes_weights_i(const int32_t* weight_index, double* weights, double cal,
+                                      const toast_interval_t* intervals, int64_t n_intervals, int64_t n_det,
+                                      int64_t n_samp, void* stream) {
+    using namespace toastb200;
+    REQUIRE_DIMS(n_det, n_samp);
+    if (n_det > 0 && n_intervals > 0) REQUIRE(weights);
+    WorkList wl;
+    int rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    if (rc != TOAST_OK) return rc;
+    cudaError_t e = launch_stokes_weights_i(wl, weight_index, weights, cal, n_det, n_samp, (cudaStream_t)stream);
+    if (e != cudaSuccess) return cuda_fail(e, "stokes_weights_i launch");
+    return ok();
+}
+
+extern "C" int toast_noise_weight(const int32_t* data_index, double* det_data, const double* det_weights,
+                                  const toast_interval_t* intervals, int64_t n_intervals, int64_t n_det, int64_t n_samp,
+                                  void* stream) {
+    using namespace toastb200;
+    REQUIRE_DIMS(n_det, n_samp);
+    if (n_det > 0 && n_intervals > 0) {
+        REQUIRE(det_data);
+        REQUIRE(det_weights);
+    }
+    WorkList wl;
+    int rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    if (rc != TOAST_OK) return rc;
+    cudaError_t e = launch_noise_weight(wl, data_index, det_data, det_weights, n_det, n_samp, (cudaStream_t)stream);
+    if (e != cudaSuccess) return cuda_fail(e, "noise_weight launch");
+    return ok();
+}
+
+extern "C" int toast_template_offset_add_to_signal(int64_t step_length, const int64_t* amp_offset,
+                                                   const double* amplitudes, const int32_t* data_index,
+                                                   double* det_data, const toast_interval_t* intervals,
+                                                   int64_t n_intervals, int64_t n_det, int64_t n_samp, void* stream) {
+    using namespace toastb200;
+    REQUIRE_DIMS(n_det, n_samp);
+    if (n_det > 0 && n_intervals > 0) {
+        REQUIRE(amp_offset);
+        REQUIRE(amplitudes);
+        REQUIRE(det_data);
+    }
+    WorkList wl;
+    int rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    if (rc != TOAST_OK) return rc;
+    OffsetViews v;
+    rc = get_offset_views(intervals, n_intervals, step_length, &v);
+    if (rc != TOAST_OK) return rc;
+    cudaError_t e = launch_offset_add(wl, v, amp_offset, amplitudes, data_index, det_data, n_det, n_samp,
+                                      (cudaStream_t)stream);
+    if (e != cudaSuccess) return cuda_fail(e, "template_offset_add_to_signal launch");
+    return ok();
+}
+
+extern "C" int toast_template_offset_project_signal(int64_t step_length, const int64_t* amp_offset, double* amplitudes,
+                                                    const int32_t* data_index, const double* det_data,
+                                                    const int32_t* flag_index, const uint8_t* det_flags,
+                                                    uint8_t det_flag_mask, const toast_interval_t* intervals,
+                                                    int64_t n_intervals, int64_t n_det, int64_t n_samp, void* stream) {
+    using namespace toastb200;
+    REQUIRE_DIMS(n_det, n_samp);
+    if (n_det > 0 && n_intervals > 0) {
+        REQUIRE(amp_offset);
+        REQUIRE(amplitudes);
+        REQUIRE(det_data);
+    }
+    WorkList wl;
+    int rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    if (rc != TOAST_OK) return rc;
+    OffsetViews v;
+    rc = get_offset_views(intervals, n_intervals, step_length, &v);
+    if (rc != TOAST_OK) return rc;
+    cudaError_t e = launch_offset_project(wl, v, amp_offset, amplitudes, data_index, det_data, flag_index, det_flags,
+                                          det_flag_mask, n_det, n_samp, (cudaStream_t)stream);
+    if (e != cudaSuccess) return cuda_fail(e, "template_offset_project_signal launch");
+    return ok();
+}
+
+extern "C" int toast_template_offset_apply_diag_precond(const double* offset_var, const double* amp_in,
+                                                        double* amp_out, int64_t n_amp, void* stream) {
+    using namespace toastb200;
+    if (n_amp < 0) return fail(TOAST_EINVAL, "n_amp = %lld < 0", (long long)n_amp);
+    if (n_amp > 0) {
+        REQUIRE(offset_var);
+        REQUIRE(amp_in);
+        REQUIRE(amp_out);
+    }
+    cudaError_t e = launch_precond(offset_var, amp_in, amp_out, n_amp, (cudaStream_t)stream);
+    if (e != cudaSuccess) return cuda_fail(e, "template_offset_apply_diag_precond launch");
     return ok();
 }

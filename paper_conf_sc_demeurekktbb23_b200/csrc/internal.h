@@ -91,6 +91,27 @@ cudaError_t launch_pointing_to_map(const WorkList& wl, const FusedArgs& a, unsig
 cudaError_t launch_pointing_to_tod(const WorkList& wl, const FusedArgs& a, unsigned long long* sched,
                                    cudaStream_t st);
 
+// Offset-template views (reading O1): per interval, its first sample and the index of its
+// first amplitude relative to the detector's amp_offset.
+struct OffsetViews {
+    const int64_t* iv_first;   // device [n_intervals]
+    const int64_t* view_base;  // device [n_intervals]
+    int step;
+};
+
+cudaError_t launch_stokes_weights_i(const WorkList& wl, const int32_t* weight_index, double* weights, double cal,
+                                    int64_t n_det, int64_t n_samp, cudaStream_t st);
+cudaError_t launch_noise_weight(const WorkList& wl, const int32_t* data_index, double* det_data,
+                                const double* det_weights, int64_t n_det, int64_t n_samp, cudaStream_t st);
+cudaError_t launch_offset_add(const WorkList& wl, const OffsetViews& v, const int64_t* amp_offset,
+                              const double* amplitudes, const int32_t* data_index, double* det_data, int64_t n_det,
+                              int64_t n_samp, cudaStream_t st);
+cudaError_t launch_offset_project(const WorkList& wl, const OffsetViews& v, const int64_t* amp_offset,
+                                  double* amplitudes, const int32_t* data_index, const double* det_data,
+                                  const int32_t* flag_index, const uint8_t* det_flags, uint8_t det_flag_mask,
+                                  int64_t n_det, int64_t n_samp, cudaStream_t st);
+cudaError_t launch_precond(const double* var, const double* in, double* out, int64_t n, cudaStream_t st);
+
 // A device counter for dynamic work distribution (zeroed on the stream before each use).
 unsigned long long* sched_counter(int* err);
 

@@ -446,3 +446,55 @@ def test_fused_pointing_to_tod(case, mode):
     assert len(bad[0]) <= 1e-6 * n_in
     out = ~np.array(_in_mask(w.intervals, w.n_det, w.n_samp))
     np.testing.assert_array_equal(got[out], w.det_data[out])  # out-of-interval samples untouched
+
+
+# ----------------------------------------------------------------------------- f2, f4
+
+NEXT_IVS = [(3, 40_002), (40_100, 40_100), (41_000, 99_998)]
+
+
+def test_stokes_weights_i_and_noise_weight_gpu():
+    n_det, n_samp = 5, 100_000
+    wg = torch.full((n_det, n_samp), -1.0, dtype=torch.float64, device=DEV)
+    binding.stokes_weights_i(wg, 1.25, NEXT_IVS)
+    ref = np.full((n_det, n_samp), -1.0)
+    oracle.stokes_weights_i(ref, 1.25, NEXT_IVS, n_det)
+    np.testing.assert_array_equal(wg.cpu().numpy(), ref)
+    rng = np.random.default_rng(91)
+    tod = rng.normal(size=(n_det, n_samp)); dwt = rng.uniform(0.1, 3, n_det)
+    ref = tod.copy(); oracle.noise_weight(ref, dwt, NEXT_IVS)
+    tg = _cuda(tod, torch.float64)
+    binding.noise_weight(tg, _cuda(dwt, torch.float64), NEXT_IVS)
+    np.testing.assert_array_equal(tg.cpu().numpy(), ref)  # one IEEE multiply: bit-exact
+
+
+@pytest.mark.parametrize("step", [1, 37, 256, 1000])
+def test_template_offsets_gpu(step):
+    n_det, n_samp = 6, 100_000
+    n_amp = oracle.offset_amplitude_counts(NEXT_IVS, step)
+    amp_offset = (np.arange(n_det, dtype=np.int64) * n_amp)[::-1].copy()  # permuted detector blocks
+    rng = np.random.default_rng(92 + step)
+    amps = rng.normal(size=n_det * n_amp)
+    tod = rng.normal(size=(n_det, n_samp))
+    flags = (rng.random((n_det, n_samp)) < 0.05).astype(np.uint8) * 2
+    # add_to_signal: one add per sample, bit-exact
+    ref = tod.copy(); oracle.template_offset_add_to_signal(step, amp_offset, amps, ref, NEXT_IVS)
+    tg = _cuda(tod, torch.float64)
+    binding.template_offset_add_to_signal(step, _cuda(amp_offset, torch.int64), _cuda(amps, torch.float64), tg,
+                                          NEXT_IVS)
+    np.testing.assert_array_equal(tg.cpu().numpy(), ref)
+    # project_signal: sums in a different order -> 1e-12 of the sum of |terms|
+    refa = np.zeros(n_det * n_amp)
+    oracle.template_offset_project_signal(step, amp_offset, refa, tod, NEXT_IVS, det_flags=flags, det_flag_mask=2)
+    absa = np.zeros(n_det * n_amp)
+    oracle.template_offset_project_signal(step, amp_offset, absa, np.abs(tod), NEXT_IVS, det_flags=flags,
+                                          det_flag_mask=2)
+    ag = torch.zeros(n_det * n_amp, dtype=torch.float64, device=DEV)
+    binding.template_offset_project_signal(step, _cuda(amp_offset, torch.int64), ag, _cuda(tod, torch.float64),
+                                           NEXT_IVS, det_flags=_cuda(flags, torch.uint8), det_flag_mask=2)
+    assert np.all(np.abs(ag.cpu().numpy() - refa) <= 1e-12 * absa + (absa == 0) * 0.0)
+    # diagonal preconditioner: one multiply, bit-exact
+    var = rng.uniform(0.1, 2, n_det * n_amp)
+    out = torch.zeros(n_det * n_amp, dtype=torch.float64, device=DEV)
+    binding.template_offset_apply_diag_precond(_cuda(var, torch.float64), ag, out)
+    np.testing.assert_array_equal(out.cpu().numpy(), oracle.template_offset_apply_diag_precond(var, ag.cpu().numpy()))
