@@ -39,7 +39,13 @@ static __constant__ double kAtanQ[11] = {
 };
 
 constexpr double kTanPi8 = 0.41421356237309504880;
-static __constant__ double kHalfTurns[9] = {0.0, 0.5, 1.0, 1.5, 2.0, 2.5, 3.0, 3.5, 4.0};  // k / 2
+// Constants whose low word is non-zero are kept in the constant bank so that the fp64
+// instructions take them as c[][] operands: written as literals, the compiler re-materialises
+// them with two UMOVs per use inside the hot loop once the uniform registers run out.
+static __constant__ double kC[3] = {kTanPi8, 1e-100, 2.0 / 3.0};
+#define TB_TAN_PI8 (::toastb200::kC[0])
+#define TB_TINY (::toastb200::kC[1])
+#define TB_TWO_THIRD (::toastb200::kC[2])
 
 // 1/x for finite x > 0 (no IEEE rounding guarantee; <= ~1 ulp): MUFU seed + 2 Newton steps.
 __device__ __forceinline__ double fast_rcp(double x) {
@@ -74,11 +80,11 @@ __device__ __forceinline__ QtPrep qt_prepare(double x, double y) {
     const bool swap = ay > ax;
     const double mx = swap ? ay : ax;
     const double mn = swap ? ax : ay;
-    const bool big = mn > kTanPi8 * mx;
+    const bool big = mn > TB_TAN_PI8 * mx;
     const double beta = big ? 1.0 : 0.0;
     QtPrep q;
     q.num = fma(-beta, mx, mn);
-    q.den = fma(beta, mn, mx) + 1e-100;  // x = y = 0 -> t = 0; changes nothing for den > 1e-84
+    q.den = fma(beta, mn, mx) + TB_TINY;  // x = y = 0 -> t = 0; changes nothing for den > 1e-84
     // K in units of half a quarter turn; S = (-1)^(swap + x<0 + y<0)
     int kk = big ? 1 : 0;
     kk = swap ? 2 - kk : kk;
@@ -109,8 +115,12 @@ __device__ __forceinline__ double qt_finish(const QtPrep& q, double t) {
     o = fma(o, s2, kAtanQ[1]);
     e = fma(e, s2, kAtanQ[0]);
     const double p = fma(o, s, e);
-    const double tau = t * p;
-    double tt = fma(q.neg ? -1.0 : 1.0, tau, kHalfTurns[q.kk]);
+    // tt = K/2 + S t P: the sign S is applied to t by flipping its sign bit (integer op), and
+    // K/2 is built exactly as (2^51 + K/2) - 2^51 (the ulp of 2^51 is 1/2), so the octant
+    // offset costs one DADD instead of a per-lane (divergent) constant-table load.
+    const double st = __hiloint2double(__double2hiint(t) ^ (q.neg ? (int)0x80000000 : 0), __double2loint(t));
+    const double half_k = __hiloint2double(0x43200000, q.kk) - 2251799813685248.0;
+    double tt = fma(st, p, half_k);
     if (tt >= 4.0) tt = 0.0;
     return tt;
 }
@@ -258,7 +268,7 @@ template <bool NEST, typename I>
 __device__ __forceinline__ int64_t loc2pix(const HealpixGeom& g, double dz, double tt, double dx, double dy) {
     const double za = fabs(dz);
     const I nside = (I)g.nside;
-    if (za <= kTwoThird) {  // equatorial belt
+    if (za <= TB_TWO_THIRD) {  // equatorial belt
         const double temp1 = __dmul_rn(g.dnside, __dadd_rn(0.5, tt));
         const double temp2 = __dmul_rn(__dmul_rn(g.dnside, dz), 0.75);
         const I jp = (I)__dsub_rn(temp1, temp2);  // ascending edge line
@@ -331,7 +341,7 @@ template <bool NEST>
 __device__ __forceinline__ int loc2pix32(const HealpixGeom& g, double dz, double tt, double dx, double dy) {
     const double za = fabs(dz);
     const int nside = (int)g.nside;
-    if (za <= kTwoThird) {
+    if (za <= TB_TWO_THIRD) {
         const double temp1 = __dmul_rn(g.dnside, __dadd_rn(0.5, tt));
         const double temp2 = __dmul_rn(__dmul_rn(g.dnside, dz), 0.75);
         const int jp = floor_nonneg(__dsub_rn(temp1, temp2));
@@ -410,10 +420,10 @@ __device__ __forceinline__ void cos_sin_2psi(double bx, double by, double& c2, d
 __device__ __forceinline__ double lon_pol(double dx, double dy, double bx, double by, double& c2, double& s2) {
     const QtPrep q = qt_prepare(dx, dy);
     const double bx2 = bx * bx;
-    const double r = fma(by, by, bx2) + 1e-100;
+    const double r = fma(by, by, bx2) + TB_TINY;
     const double inv = fast_rcp(q.den * r);
     const double invr = q.den * inv;
-    c2 = fma(-by, by, bx2 + 1e-100) * invr;
+    c2 = fma(-by, by, bx2 + TB_TINY) * invr;
     s2 = 2.0 * bx * by * invr;
     return qt_finish(q, q.num * (r * inv));
 }

@@ -192,8 +192,9 @@ __device__ __forceinline__ void load_slot(Slot<P>& sl, const FusedArgs& a, int64
     const double eps = __ldg(&a.epsilon[dd]);
     const double scale = __ldg(&a.det_scale[dd]);
     sl.etacal = (1.0 - eps) / (1.0 + eps) * a.cal;
-    sl.s_cal = scale * a.cal;
-    sl.s_eta = scale * sl.etacal;
+    // a lane without a detector contributes exactly 0 (aggregate() adds unconditionally)
+    sl.s_cal = ok ? scale * a.cal : 0.0;
+    sl.s_eta = ok ? scale * sl.etacal : 0.0;
     sl.run_pix = -1;
     sl.run_loc = -1;
     sl.last_sm = -1;
@@ -259,35 +260,37 @@ __device__ __forceinline__ void det_sample(Slot<typename PixT<WIDE>::T>& sl, con
     }
     // A4 contribution of this det-sample; it is folded into the lane's run by aggregate()
     // one sample LATER, so that work overlaps the shared-memory loads of the next sample.
-    // Det-flagged samples keep their pixel (they mark hit submaps, as A2 does) but add 0.
+    // Det-flagged samples keep their pixel (they mark hit submaps, as A2 does) but add 0;
+    // so does every sample without a pixel (aggregate() adds unconditionally).
     sl.pend_pix = pix;
-    sl.p0 = dflag ? 0.0 : tod * sl.s_cal;
+    const double tz = (dflag || (DEBUG && !pixelise)) ? 0.0 : tod;
+    sl.p0 = tz * sl.s_cal;
     if (NNZ == 3) {
-        const double t = dflag ? 0.0 : tod * sl.s_eta;
+        const double t = tz * sl.s_eta;
         sl.p1 = t * c2;
         sl.p2 = t * s2;
     }
 }
 
 // Fold the pending contribution into the run (run-length aggregation along time).  Lanes
-// without a pixel (no detector / flagged sample) have pend_pix = -1 and never touch their run.
+// without a pixel (no detector / flagged sample) have pend_pix = -1 and never start a run.
+// A pending sample without a pixel carries zero contributions, so the add is unconditional
+// (one branch less per det-sample); pend_pix is not reset here because det_sample() always
+// overwrites it right after (the end-of-item call is followed by the final flush).
 template <int NNZ, typename P>
 __device__ __forceinline__ void aggregate(Slot<P>& sl, const FusedArgs& a) {
-    if (sl.pend_pix >= 0) {
-        if (sl.pend_pix != sl.run_pix) {
+    if (sl.pend_pix >= 0 && sl.pend_pix != sl.run_pix) {
 #ifndef TB_X_NOFLUSH
-            if (sl.run_pix >= 0) flush<NNZ, P>(sl.run_pix, sl.run_loc, sl.r0, sl.r1, sl.r2, a);
+        if (sl.run_pix >= 0) flush<NNZ, P>(sl.run_pix, sl.run_loc, sl.r0, sl.r1, sl.r2, a);
 #endif
-            sl.run_pix = sl.pend_pix;
-            sl.run_loc = start_run<P>(sl.pend_pix, a, sl.last_sm);
-            sl.r0 = sl.r1 = sl.r2 = 0.0;
-        }
-        sl.r0 += sl.p0;
-        if (NNZ == 3) {
-            sl.r1 += sl.p1;
-            sl.r2 += sl.p2;
-        }
-        sl.pend_pix = -1;
+        sl.run_pix = sl.pend_pix;
+        sl.run_loc = start_run<P>(sl.pend_pix, a, sl.last_sm);
+        sl.r0 = sl.r1 = sl.r2 = 0.0;
+    }
+    sl.r0 += sl.p0;
+    if (NNZ == 3) {
+        sl.r1 += sl.p1;
+        sl.r2 += sl.p2;
     }
 }
 
@@ -457,9 +460,10 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
         }
         __syncwarp();
 
+        unsigned bit = 1u;  // 1 << k
 #pragma unroll kKUnroll
-        for (int k = 0; k < cur.nb; ++k) {
-            const bool pixelise = (pmask >> k) & 1u;
+        for (int k = 0; k < cur.nb; ++k, bit <<= 1) {
+            const bool pixelise = pmask & bit;
             if (!DEBUG && !pixelise) continue;  // shared-flagged sample: nothing to add (uniform)
             double x[12];
 #pragma unroll
@@ -474,7 +478,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
             for (int j = 0; j < DPL; ++j) {
                 const int row = lane + 32 * j;
                 tod[j] = rb.tod[row][k];
-                dflag[j] = (fmask[j] >> k) & 1u;
+                dflag[j] = fmask[j] & bit;
             }
             // fold the previous sample while those shared-memory loads are in flight
 #pragma unroll

@@ -14,14 +14,27 @@ namespace {
 
 constexpr unsigned kFullMask = 0xffffffffu;
 
+// IDX = false: no row-index array (the common case) — no branch between the loads, so the
+// kDT detectors' loads issue back to back.
+template <bool IDX>
 __device__ __forceinline__ int64_t row_or(const int32_t* __restrict__ index, int64_t d) {
-    return index ? (int64_t)__ldg(&index[d]) : d;
+    return (IDX && index) ? (int64_t)__ldg(&index[d]) : d;
 }
 
-dim3 grid2(const WorkList& wl, int64_t n_det) {
-    return dim3((unsigned)std::min<int64_t>(wl.n_chunks, 0x7fffffff), (unsigned)std::min<int64_t>(n_det, 65535), 1);
+// A CTA covers kDT detectors of one chunk: each thread keeps kDT independent loads in flight
+// (one (chunk, detector) per CTA left a 2 KB CTA with a dependent chunk-descriptor load in
+// front of one 8-byte load per thread — latency-bound at ~40 % of HBM bandwidth).
+#ifndef TB_TPL_DT
+#define TB_TPL_DT 4  // measured best of 1/4/8 (noise_weight 94 %, projection 2x faster than 8)
+#endif
+constexpr int kDT = TB_TPL_DT;
+
+dim3 grid_dt(const WorkList& wl, int64_t n_det) {
+    return dim3((unsigned)std::min<int64_t>(wl.n_chunks, 0x7fffffff),
+                (unsigned)std::min<int64_t>((n_det + kDT - 1) / kDT, 65535), 1);
 }
 
+template <bool IDX>
 __global__ void __launch_bounds__(kChunk) stokes_weights_i_kernel(const Chunk* __restrict__ chunks, int64_t n_chunks,
                                                                   const int32_t* __restrict__ weight_index,
                                                                   double* __restrict__ weights, double cal,
@@ -30,10 +43,15 @@ __global__ void __launch_bounds__(kChunk) stokes_weights_i_kernel(const Chunk* _
         const Chunk ch = chunks[c];
         if ((int)threadIdx.x >= ch.count) continue;
         const int64_t s = ch.first + threadIdx.x;
-        for (int64_t d = blockIdx.y; d < n_det; d += gridDim.y) weights[row_or(weight_index, d) * n_samp + s] = cal;
+        for (int64_t d0 = (int64_t)blockIdx.y * kDT; d0 < n_det; d0 += (int64_t)gridDim.y * kDT) {
+#pragma unroll
+            for (int j = 0; j < kDT; ++j)
+                if (d0 + j < n_det) weights[row_or<IDX>(weight_index, d0 + j) * n_samp + s] = cal;
+        }
     }
 }
 
+template <bool IDX>
 __global__ void __launch_bounds__(kChunk) noise_weight_kernel(const Chunk* __restrict__ chunks, int64_t n_chunks,
                                                               const int32_t* __restrict__ data_index,
                                                               double* __restrict__ det_data,
@@ -43,18 +61,23 @@ __global__ void __launch_bounds__(kChunk) noise_weight_kernel(const Chunk* __res
         const Chunk ch = chunks[c];
         if ((int)threadIdx.x >= ch.count) continue;
         const int64_t s = ch.first + threadIdx.x;
-        for (int64_t d = blockIdx.y; d < n_det; d += gridDim.y)
-            det_data[row_or(data_index, d) * n_samp + s] *= __ldg(&det_weights[d]);
+        for (int64_t d0 = (int64_t)blockIdx.y * kDT; d0 < n_det; d0 += (int64_t)gridDim.y * kDT) {
+            int64_t o[kDT];
+            double v[kDT];
+#pragma unroll
+            for (int j = 0; j < kDT; ++j) {
+                o[j] = d0 + j < n_det ? row_or<IDX>(data_index, d0 + j) * n_samp + s : -1;
+                v[j] = o[j] >= 0 ? det_data[o[j]] * __ldg(&det_weights[d0 + j]) : 0.0;
+            }
+#pragma unroll
+            for (int j = 0; j < kDT; ++j)
+                if (o[j] >= 0) det_data[o[j]] = v[j];
+        }
     }
 }
 
 // Amplitude of (d, s) under reading O1: amp_offset[d] + view_base[iv] + (s - iv_first[iv]) / step.
-__device__ __forceinline__ int64_t offset_index(const OffsetViews& v, const int64_t* __restrict__ amp_offset,
-                                                int64_t d, const Chunk& ch, int64_t s) {
-    const int64_t first = __ldg(&v.iv_first[ch.interval]);
-    return __ldg(&amp_offset[d]) + __ldg(&v.view_base[ch.interval]) + (int64_t)((int)(s - first) / v.step);
-}
-
+template <bool IDX>
 __global__ void __launch_bounds__(kChunk) offset_add_kernel(const Chunk* __restrict__ chunks, int64_t n_chunks,
                                                             OffsetViews v, const int64_t* __restrict__ amp_offset,
                                                             const double* __restrict__ amplitudes,
@@ -65,14 +88,30 @@ __global__ void __launch_bounds__(kChunk) offset_add_kernel(const Chunk* __restr
         const Chunk ch = chunks[c];
         if ((int)threadIdx.x >= ch.count) continue;
         const int64_t s = ch.first + threadIdx.x;
-        for (int64_t d = blockIdx.y; d < n_det; d += gridDim.y)
-            det_data[row_or(data_index, d) * n_samp + s] += __ldg(&amplitudes[offset_index(v, amp_offset, d, ch, s)]);
+        const int64_t rel = __ldg(&v.view_base[ch.interval]) +
+                            (int64_t)((int)(s - __ldg(&v.iv_first[ch.interval])) / v.step);
+        for (int64_t d0 = (int64_t)blockIdx.y * kDT; d0 < n_det; d0 += (int64_t)gridDim.y * kDT) {
+            int64_t o[kDT];
+            double t[kDT], a[kDT];
+#pragma unroll
+            for (int j = 0; j < kDT; ++j) {
+                const bool ok = d0 + j < n_det;
+                o[j] = ok ? row_or<IDX>(data_index, d0 + j) * n_samp + s : -1;
+                t[j] = ok ? det_data[o[j]] : 0.0;
+                a[j] = ok ? __ldg(&amplitudes[__ldg(&amp_offset[d0 + j]) + rel]) : 0.0;
+            }
+#pragma unroll
+            for (int j = 0; j < kDT; ++j)
+                if (o[j] >= 0) det_data[o[j]] = t[j] + a[j];
+        }
     }
 }
 
 // Projection: the samples of one step are consecutive, so a warp (32 consecutive samples of
 // one detector) holds runs of equal amplitude index; each run is summed by a segmented
-// shuffle scan and its last lane issues ONE fp64 red.
+// shuffle scan and its last lane issues ONE fp64 red.  The kDT detectors' loads are issued
+// together, then reduced one detector at a time.
+template <bool IDX>
 __global__ void __launch_bounds__(kChunk) offset_project_kernel(
     const Chunk* __restrict__ chunks, int64_t n_chunks, OffsetViews v, const int64_t* __restrict__ amp_offset,
     double* __restrict__ amplitudes, const int32_t* __restrict__ data_index, const double* __restrict__ det_data,
@@ -84,29 +123,55 @@ __global__ void __launch_bounds__(kChunk) offset_project_kernel(
         if ((int)(threadIdx.x & ~31u) >= ch.count) continue;  // whole warp past the chunk
         const bool in = (int)threadIdx.x < ch.count;
         const int64_t s = ch.first + threadIdx.x;
-        for (int64_t d = blockIdx.y; d < n_det; d += gridDim.y) {
-            int64_t key = -1 - lane;
-            double val = 0.0;
-            if (in) {
-                const bool fl = det_flags && (__ldg(&det_flags[row_or(flag_index, d) * n_samp + s]) & det_flag_mask);
-                if (!fl) {
-                    key = offset_index(v, amp_offset, d, ch, s);
-                    val = __ldg(&det_data[row_or(data_index, d) * n_samp + s]);
+        // amplitude index relative to the detector's amp_offset; runs are detector-independent
+        const int64_t rel = __ldg(&v.view_base[ch.interval]) +
+                            (int64_t)((int)(s - __ldg(&v.iv_first[ch.interval])) / v.step);
+        const int64_t rprev = __shfl_up_sync(kFullMask, rel, 1);
+        for (int64_t d0 = (int64_t)blockIdx.y * kDT; d0 < n_det; d0 += (int64_t)gridDim.y * kDT) {
+            double val[kDT];
+            unsigned okm = 0u;  // bit j: this lane contributes to detector d0 + j
+#pragma unroll
+            for (int j = 0; j < kDT; ++j) {
+                val[j] = 0.0;
+                if (in && d0 + j < n_det) {
+                    // both loads issued unconditionally (the TOD load must not wait for the flag)
+                    const bool fl =
+                        det_flags && (__ldg(&det_flags[row_or<IDX>(flag_index, d0 + j) * n_samp + s]) & det_flag_mask);
+#ifdef TB_PROJ_COND
+                    if (!fl) {
+                        val[j] = __ldg(&det_data[row_or<IDX>(data_index, d0 + j) * n_samp + s]);
+                        okm |= 1u << j;
+                    }
+#else
+                    const double t = __ldg(&det_data[row_or<IDX>(data_index, d0 + j) * n_samp + s]);
+                    if (!fl) {
+                        val[j] = t;
+                        okm |= 1u << j;
+                    }
+#endif
                 }
             }
-            const int64_t kprev = __shfl_up_sync(kFullMask, key, 1);
-            const unsigned heads = __ballot_sync(kFullMask, lane == 0 || kprev != key);
-            const int start = 31 - __clz(heads & (kFullMask >> (31 - lane)));
-            const int depth = lane - start;
 #pragma unroll
-            for (int off = 1; off < 32; off <<= 1) {
-                const bool need = depth >= off;
-                if (!__any_sync(kFullMask, need)) break;
-                const double t = __shfl_up_sync(kFullMask, val, off);
-                if (need) val += t;
+            for (int j = 0; j < kDT; ++j) {
+                if (d0 + j >= n_det) break;
+                // a run = consecutive lanes with equal rel that contribute
+                const bool ok = (okm >> j) & 1u;
+                const bool okp = __shfl_up_sync(kFullMask, ok, 1);
+                const bool head = lane == 0 || rprev != rel || !okp || !ok;
+                const unsigned heads = __ballot_sync(kFullMask, head);
+                const int start = 31 - __clz(heads & (kFullMask >> (31 - lane)));
+                const int depth = lane - start;
+                double x = val[j];
+#pragma unroll
+                for (int off = 1; off < 32; off <<= 1) {
+                    const bool need = depth >= off;
+                    if (!__any_sync(kFullMask, need)) break;
+                    const double t = __shfl_up_sync(kFullMask, x, off);
+                    if (need) x += t;
+                }
+                const bool tail = lane == 31 || ((heads >> (lane + 1)) & 1u);
+                if (tail && ok) atomicAdd(&amplitudes[__ldg(&amp_offset[d0 + j]) + rel], x);
             }
-            const bool tail = lane == 31 || ((heads >> (lane + 1)) & 1u);
-            if (tail && key >= 0) atomicAdd(&amplitudes[key], val);
         }
     }
 }
@@ -122,7 +187,7 @@ __global__ void precond_kernel(const double* __restrict__ var, const double* __r
 cudaError_t launch_stokes_weights_i(const WorkList& wl, const int32_t* weight_index, double* weights, double cal,
                                     int64_t n_det, int64_t n_samp, cudaStream_t st) {
     if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
-    stokes_weights_i_kernel<<<grid2(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, weight_index, weights, cal,
+    (weight_index ? stokes_weights_i_kernel<true> : stokes_weights_i_kernel<false>)<<<grid_dt(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, weight_index, weights, cal,
                                                                   n_det, n_samp);
     return cudaGetLastError();
 }
@@ -130,7 +195,7 @@ cudaError_t launch_stokes_weights_i(const WorkList& wl, const int32_t* weight_in
 cudaError_t launch_noise_weight(const WorkList& wl, const int32_t* data_index, double* det_data,
                                 const double* det_weights, int64_t n_det, int64_t n_samp, cudaStream_t st) {
     if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
-    noise_weight_kernel<<<grid2(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, data_index, det_data,
+    (data_index ? noise_weight_kernel<true> : noise_weight_kernel<false>)<<<grid_dt(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, data_index, det_data,
                                                               det_weights, n_det, n_samp);
     return cudaGetLastError();
 }
@@ -139,7 +204,7 @@ cudaError_t launch_offset_add(const WorkList& wl, const OffsetViews& v, const in
                               const double* amplitudes, const int32_t* data_index, double* det_data, int64_t n_det,
                               int64_t n_samp, cudaStream_t st) {
     if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
-    offset_add_kernel<<<grid2(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, v, amp_offset, amplitudes,
+    (data_index ? offset_add_kernel<true> : offset_add_kernel<false>)<<<grid_dt(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, v, amp_offset, amplitudes,
                                                             data_index, det_data, n_det, n_samp);
     return cudaGetLastError();
 }
@@ -149,7 +214,7 @@ cudaError_t launch_offset_project(const WorkList& wl, const OffsetViews& v, cons
                                   const int32_t* flag_index, const uint8_t* det_flags, uint8_t det_flag_mask,
                                   int64_t n_det, int64_t n_samp, cudaStream_t st) {
     if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
-    offset_project_kernel<<<grid2(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, v, amp_offset, amplitudes,
+    (data_index || flag_index ? offset_project_kernel<true> : offset_project_kernel<false>)<<<grid_dt(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, v, amp_offset, amplitudes,
                                                                 data_index, det_data, flag_index, det_flags,
                                                                 det_flag_mask, n_det, n_samp);
     return cudaGetLastError();
