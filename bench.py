@@ -344,7 +344,8 @@ def main():
                            "step": "zero map + toast_pointing_to_map" + (
                                (" + all_reduce(hit submaps, MAX) + packed all_reduce(map)" if packed
                                 else " + all_reduce(map)") if world > 1 else ""),
-                           "allreduce_bytes_per_step": reduced[0]},
+                           "allreduce_bytes_per_step": reduced[0],
+                           "staging": binding.last_fused_path()},
                 "clocks": clocks, "gpu_launches": args.steps, "roofline": roofline}
         if e2e is not None:
             line["e2e"] = e2e

@@ -45,6 +45,7 @@ def load():
     L = ctypes.CDLL(path)
     L.toast_last_error.restype = ctypes.c_char_p
     L.toast_version.restype = ctypes.c_char_p
+    L.toast_last_fused_path.restype = ctypes.c_char_p
     L.toast_release.restype = I32
     L.toast_pointing_detector.argtypes = [P, P, P, P, P, I64, P, U8, I64, I64, P]
     L.toast_pixels_healpix.argtypes = [P, P, P, U8, P, P, P, I64, P, I64, I64, I32, I64, I64, P]
@@ -70,7 +71,7 @@ def load():
     return L
 
 
-EXPORTED = ("toast_last_error", "toast_version", "toast_release", "toast_pointing_detector", "toast_pixels_healpix",
+EXPORTED = ("toast_last_error", "toast_version", "toast_last_fused_path", "toast_release", "toast_pointing_detector", "toast_pixels_healpix",
             "toast_stokes_weights_iqu", "toast_build_noise_weighted", "toast_scan_map", "toast_pointing_to_map",
             "toast_pointing_to_tod", "toast_stokes_weights_i", "toast_noise_weight",
             "toast_template_offset_add_to_signal", "toast_template_offset_project_signal",
@@ -79,6 +80,11 @@ EXPORTED = ("toast_last_error", "toast_version", "toast_release", "toast_pointin
 
 def version() -> str:
     return load().toast_version().decode()
+
+
+def last_fused_path() -> str:
+    """How the last pointing_to_map call on this thread staged its inputs ("tma" / "cp.async (...)")."""
+    return load().toast_last_fused_path().decode()
 
 
 def release() -> None:

@@ -212,6 +212,8 @@ const char* toast_last_error(void) { return g_last_error.c_str(); }
 
 const char* toast_version(void) { return "toastb200 0.1.0 (sm_100a)"; }
 
+const char* toast_last_fused_path(void) { return last_fused_path(); }
+
 int toast_release(void) {
     std::lock_guard<std::mutex> lk(g_cache_mu);
     int cur = 0;

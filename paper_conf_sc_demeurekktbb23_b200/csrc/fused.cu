@@ -25,9 +25,12 @@
 //   * Map accumulation is RUN-LENGTH aggregated per lane along time: consecutive samples of
 //     one detector that fall in the same pixel are summed in registers and flushed with one
 //     fp64 `red` per Stokes component when the pixel changes (no shuffles at all).
+#include <cuda.h>  // CUtensorMap (the encoder is fetched through the runtime; no -lcuda)
 #include <cuda_runtime.h>
+#include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <cstring>
 #include <mutex>
 
 #include "device_math.cuh"
@@ -109,6 +112,82 @@ __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wai
 __device__ __forceinline__ void cp_async_bytes(uint8_t* dst, const uint8_t* p, int n, int w) {
     const uint8_t* w0 = reinterpret_cast<const uint8_t*>(reinterpret_cast<uintptr_t>(p) & ~uintptr_t(3));
     if (w0 + 4 * w < p + n) cp_async4(dst + 4 * w, w0 + 4 * w);
+}
+
+// ----------------------------------------------------------------------------- TMA path
+// When the inputs satisfy the tensor-memory-accelerator constraints (n_samp % 16 == 0 and
+// 16-byte aligned arrays), lane 0 moves a whole block with five
+// bulk tensor copies that complete on a per-buffer mbarrier, instead of 32 lanes issuing
+// ~30 cp.async each with 64-bit address arithmetic.  The TOD tile [32 det][16 samples] lands
+// 128-byte-swizzled (row r's 16-byte chunk c at c ^ (r & 7)), so the per-sample column read
+// tod[lane][k] is a 4-wavefront access without padding bytes.  Boxes start at multiples of 16
+// samples (a box must start 16-byte aligned in every staged row).
+struct alignas(64) TmaMaps {
+    CUtensorMap tod;   // f64 [n_det][n_samp], box {16, 32}, SWIZZLE_128B
+    CUtensorMap flg;   // u8  [n_det][n_samp], box {16, 32}
+    CUtensorMap bore;  // f64 [n_samp][4],     box {4, 16}
+    CUtensorMap hwp;   // f64 [n_samp],        box {16}
+    CUtensorMap sflg;  // u8  [n_samp],        box {16}
+};
+
+// Every TMA destination is 128-byte aligned; the 16 shared-flag bytes of a buffer share their
+// 128-byte slot with that buffer's mbarrier, so a warp's staging area is exactly 12 KB.
+struct alignas(128) SflgSlot {
+    uint8_t f[16];
+    unsigned long long mbar;
+    uint8_t pad[104];
+};
+struct alignas(1024) TmaWarpSmem {
+    double tod[2][32][16];           // 1024-aligned (the 128-byte swizzle pattern spans 1 KB)
+    uint8_t flg[2][32][16];
+    double bore[2][16][4];
+    double hwp[2][16];
+    SflgSlot sf[2];
+    double st[16][12];               // SampleState[kBlk]
+};
+static_assert(sizeof(TmaWarpSmem) == 12288, "TMA staging area: 12 KB per warp");
+
+__device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(unsigned long long* bar) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(unsigned long long* bar, unsigned bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned parity) {
+    unsigned done;
+    do {
+        asm volatile(
+            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+            : "=r"(done)
+            : "r"(smem_u32(bar)), "r"(parity)
+            : "memory");
+    } while (!done);
+}
+__device__ __forceinline__ void tma_1d(void* dst, const CUtensorMap* m, int c0, unsigned long long* bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.1d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2}], [%3];\n" ::"r"(
+            smem_u32(dst)),
+        "l"(m), "r"(c0), "r"(smem_u32(bar))
+        : "memory");
+}
+__device__ __forceinline__ void tma_2d(void* dst, const CUtensorMap* m, int c0, int c1, unsigned long long* bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], "
+        "[%4];\n" ::"r"(smem_u32(dst)),
+        "l"(m), "r"(c0), "r"(c1), "r"(smem_u32(bar))
+        : "memory");
+}
+// streamed-once TOD / det flags with an L2 evict-first hint (see evict_first_policy)
+__device__ __forceinline__ void tma_2d_stream(void* dst, const CUtensorMap* m, int c0, int c1,
+                                              unsigned long long* bar, uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1, "
+        "{%2, %3}], [%4], %5;\n" ::"r"(smem_u32(dst)),
+        "l"(m), "r"(c0), "r"(c1), "r"(smem_u32(bar)), "l"(pol)
+        : "memory");
 }
 
 // Pixel index type: 32-bit up to nside 8192 (12 nside^2 < 2^31), else 64-bit.
@@ -298,10 +377,11 @@ __device__ __forceinline__ void aggregate(Slot<P>& sl, const FusedArgs& a) {
 struct Blk {
     int64_t item;  // < 0: end of stream
     int64_t d0;
-    int64_t s0;
+    int64_t s0;     // first sample of the staged box
     int64_t s_end;  // end of the item's chunk
-    int nb;
+    int nb;         // samples processed: box indices k0 .. k0 + nb - 1
     int nrows;
+    int k0 = 0;     // TMA path: first processed box sample (boxes start at multiples of 16)
 };
 
 template <int DPL>
@@ -339,16 +419,21 @@ __device__ __forceinline__ void issue_block(RawBlock<DPL>& rb, const Blk& bk, co
     cp_async_commit();
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL>
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL, bool TMA>
 __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_kernel(const Chunk* __restrict__ chunks,
                                                                          int64_t n_chunks, FusedArgs a,
                                                                          HealpixGeom g,
-                                                                         unsigned long long* __restrict__ sched) {
+                                                                         unsigned long long* __restrict__ sched,
+                                                                         const __grid_constant__ TmaMaps tm) {
+    static_assert(!TMA || (DPL == 1 && kBlk == 16), "the TMA path stages 32 x 16 tiles");
     using P = typename PixT<WIDE>::T;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int lane = threadIdx.x & 31;
     const int wid = threadIdx.x >> 5;
+    // cp.async path: WarpSmem<DPL>; TMA path: TmaWarpSmem (1 KB-aligned, see launch_t)
     WarpSmem<DPL>& sm = reinterpret_cast<WarpSmem<DPL>*>(smem_raw)[wid];
+    TmaWarpSmem& tw = reinterpret_cast<TmaWarpSmem*>(
+        (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023))[wid];
     constexpr int kRows = 32 * DPL;
     const int64_t n_groups = (a.n_det + kRows - 1) / kRows;
     const int64_t n_items = n_chunks * n_groups;
@@ -356,6 +441,12 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
     const unsigned smask = a.shared_flag_mask;
     const bool have_dflags = a.det_flags != nullptr;
     const bool have_sflags = a.shared_flags != nullptr;
+    // TMA: bytes landing per block (full boxes, out-of-range elements zero-filled)
+    const unsigned tx_bytes = 32 * 16 * 8 + 16 * 32 + (have_dflags ? 32 * 16 : 0) +
+                              ((HWP && NNZ == 3) ? 16 * 8 : 0) + (have_sflags ? 16 : 0);
+    unsigned phase = 0u;  // TMA: bit b = parity of the next completion of mbar[b]
+    // swizzled byte offset of row `lane` in a TOD tile; sample k is at row_swz ^ (8 k)
+    const unsigned row_swz = (unsigned)lane * 128u + (((unsigned)lane & 7u) << 4);
 
     // Lane 0 fetches the NEXT item id and its chunk descriptor one item ahead (issued at
     // an item switch, consumed at the next one), so neither latency is on the critical path.
@@ -388,14 +479,50 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
         bk.s0 = first;
         bk.s_end = first + count;
         bk.nb = count < kBlk ? count : kBlk;
+        if (TMA) {
+            // TMA boxes must start on 16-byte boundaries of every staged row (measured: an odd
+            // f64 start faults), so boxes are aligned to 16 samples — the u8 flag rows need
+            // that — and a chunk's first block processes box samples k0 .. 15 only
+            bk.k0 = (int)(first & 15);
+            bk.s0 = first - bk.k0;
+            bk.nb = count < kBlk - bk.k0 ? count : kBlk - bk.k0;
+        }
         return bk;
     };
+    // Stage the raw inputs of block bk into buffer b.
+    auto issue = [&](int b, const Blk& bk) {
+        if constexpr (TMA) {
+            if (lane == 0) {
+                // the generic-proxy reads of buffer b (two blocks ago) are ordered before the
+                // async-proxy writes that refill it
+                asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+                mbar_expect_tx(&tw.sf[b].mbar, tx_bytes);
+                const uint64_t pol = evict_first_policy();
+                const int s0 = (int)bk.s0, d0 = (int)bk.d0;
+                tma_2d_stream(&tw.tod[b][0][0], &tm.tod, s0, d0, &tw.sf[b].mbar, pol);
+                if (have_dflags) tma_2d_stream(&tw.flg[b][0][0], &tm.flg, s0, d0, &tw.sf[b].mbar, pol);
+                tma_2d(&tw.bore[b][0][0], &tm.bore, 0, s0, &tw.sf[b].mbar);
+                if (HWP && NNZ == 3) tma_1d(&tw.hwp[b][0], &tm.hwp, s0, &tw.sf[b].mbar);
+                if (have_sflags) tma_1d(&tw.sf[b].f[0], &tm.sflg, s0, &tw.sf[b].mbar);
+            }
+        } else {
+            issue_block<DPL>(sm.buf[b], bk, a, have_dflags, HWP && NNZ == 3, lane);
+        }
+    };
 
+    if constexpr (TMA) {
+        if (lane == 0) {
+            mbar_init(&tw.sf[0].mbar);
+            mbar_init(&tw.sf[1].mbar);
+            asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+        }
+        __syncwarp();
+    }
     prefetch_item();
     Blk cur = take_item();
     if (cur.item < 0) return;
     prefetch_item();
-    issue_block<DPL>(sm.buf[0], cur, a, have_dflags, HWP && NNZ == 3, lane);
+    issue(0, cur);
     Slot<P> sl[DPL];
 #pragma unroll
     for (int j = 0; j < DPL; ++j) load_slot<P>(sl[j], a, cur.d0 + lane + 32 * j, lane + 32 * j < cur.nrows, cur.d0);
@@ -407,14 +534,20 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
         if (cur.s0 + kBlk < cur.s_end) {
             nxt = cur;
             nxt.s0 = cur.s0 + kBlk;
+            nxt.k0 = 0;
             nxt.nb = (nxt.s_end - nxt.s0) < kBlk ? (int)(nxt.s_end - nxt.s0) : kBlk;
         } else {
             nxt = take_item();
             if (nxt.item >= 0) prefetch_item();
         }
-        cp_async_wait_all();
-        __syncwarp();
-        if (nxt.item >= 0) issue_block<DPL>(sm.buf[p ^ 1], nxt, a, have_dflags, HWP && NNZ == 3, lane);
+        if constexpr (TMA) {
+            mbar_wait(&tw.sf[p].mbar, (phase >> p) & 1u);
+            phase ^= 1u << p;
+        } else {
+            cp_async_wait_all();
+            __syncwarp();
+        }
+        if (nxt.item >= 0) issue(p ^ 1, nxt);
 
         RawBlock<DPL>& rb = sm.buf[p];
         // per-sample state (lanes 0..15); bit k of pmask = sample k is pixelised
@@ -422,21 +555,31 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
         if (lane < kBlk) {
             double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 1.0;
             double c4 = 1.0, s4 = 0.0;
-            if (lane < cur.nb) {
-                const int soff = have_sflags ? (int)(reinterpret_cast<uintptr_t>(a.shared_flags + cur.s0) & 3) : 0;
-                const bool flagged = have_sflags && (rb.sflg[soff + lane] & smask);
-                pixelise_me = !flagged;
-                if (!flagged) {
-                    q0 = rb.bore[lane][0]; q1 = rb.bore[lane][1]; q2 = rb.bore[lane][2]; q3 = rb.bore[lane][3];
+            if (lane >= cur.k0 && lane < cur.k0 + cur.nb) {
+                bool flagged;
+                if constexpr (TMA) {
+                    flagged = have_sflags && (tw.sf[p].f[lane] & smask);
+                } else {
+                    const int soff =
+                        have_sflags ? (int)(reinterpret_cast<uintptr_t>(a.shared_flags + cur.s0) & 3) : 0;
+                    flagged = have_sflags && (rb.sflg[soff + lane] & smask);
                 }
-                if (HWP && NNZ == 3) small_sincos(4.0 * rb.hwp[lane], &s4, &c4);
+                pixelise_me = !flagged;
+                const double* bq = TMA ? tw.bore[p][lane] : rb.bore[lane];
+                if (!flagged) {
+                    q0 = bq[0]; q1 = bq[1]; q2 = bq[2]; q3 = bq[3];
+                }
+                if (HWP && NNZ == 3) small_sincos(4.0 * (TMA ? tw.hwp[p][lane] : rb.hwp[lane]), &s4, &c4);
             }
             SampleState x;
             quat_to_matrix(q0, q1, q2, q3, x.v);
             x.v[9] = c4;
             x.v[10] = s4;
             x.v[11] = 0.0;
-            sm.st[lane] = x;
+            if constexpr (TMA)
+                *reinterpret_cast<SampleState*>(tw.st[lane]) = x;
+            else
+                sm.st[lane] = x;
         }
         const unsigned pmask = __ballot_sync(0xffffffffu, pixelise_me);
         // det flags of the lane's rows -> one bit per sample (bit k: sample k is det-flagged)
@@ -446,29 +589,44 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
             fmask[j] = 0u;
             const int row = lane + 32 * j;
             if (have_dflags && row < cur.nrows) {
-                const int foff =
-                    (int)(reinterpret_cast<uintptr_t>(a.det_flags + (cur.d0 + row) * a.n_samp + cur.s0) & 3);
                 const unsigned rep = dmask * 0x01010101u;
-                unsigned bits = 0u;  // bit b: byte b of the 20-byte window is flagged
+                const unsigned keep = ((1u << cur.nb) - 1u) << cur.k0;  // nb <= 16
+                if constexpr (TMA) {
+                    const uint4 f = *reinterpret_cast<const uint4*>(tw.flg[p][row]);
+                    const unsigned fw[4] = {f.x, f.y, f.z, f.w};
+                    unsigned bits = 0u;
 #pragma unroll
-                for (int w = 0; w < 5; ++w) {
-                    const unsigned v = __vcmpne4(*reinterpret_cast<const unsigned*>(&rb.flg[row][4 * w]) & rep, 0u);
-                    bits |= ((v & 0x01010101u) * 0x01020408u >> 24 & 0xfu) << (4 * w);
+                    for (int w = 0; w < 4; ++w) {
+                        const unsigned v = __vcmpne4(fw[w] & rep, 0u);
+                        bits |= ((v & 0x01010101u) * 0x01020408u >> 24 & 0xfu) << (4 * w);
+                    }
+                    fmask[j] = bits & keep;
+                } else {
+                    const int foff =
+                        (int)(reinterpret_cast<uintptr_t>(a.det_flags + (cur.d0 + row) * a.n_samp + cur.s0) & 3);
+                    unsigned bits = 0u;  // bit b: byte b of the 20-byte window is flagged
+#pragma unroll
+                    for (int w = 0; w < 5; ++w) {
+                        const unsigned v = __vcmpne4(*reinterpret_cast<const unsigned*>(&rb.flg[row][4 * w]) & rep, 0u);
+                        bits |= ((v & 0x01010101u) * 0x01020408u >> 24 & 0xfu) << (4 * w);
+                    }
+                    fmask[j] = (bits >> foff) & keep;
                 }
-                fmask[j] = (bits >> foff) & ((cur.nb >= 32) ? 0xffffffffu : ((1u << cur.nb) - 1u));
             }
         }
         __syncwarp();
 
-        unsigned bit = 1u;  // 1 << k
+        const double* st_base = TMA ? &tw.st[0][0] : &sm.st[0].v[0];
+        const unsigned char* tod_tile = reinterpret_cast<const unsigned char*>(&tw.tod[p][0][0]);
+        unsigned bit = 1u << cur.k0;  // 1 << k
 #pragma unroll kKUnroll
-        for (int k = 0; k < cur.nb; ++k, bit <<= 1) {
+        for (int k = cur.k0; k < cur.k0 + cur.nb; ++k, bit <<= 1) {
             const bool pixelise = pmask & bit;
             if (!DEBUG && !pixelise) continue;  // shared-flagged sample: nothing to add (uniform)
             double x[12];
 #pragma unroll
             for (int i = 0; i < ((HWP && NNZ == 3) ? 12 : 10); i += 2) {
-                const double2 t2 = *reinterpret_cast<const double2*>(&sm.st[k].v[i]);
+                const double2 t2 = *reinterpret_cast<const double2*>(st_base + 12 * k + i);
                 x[i] = t2.x;
                 x[i + 1] = t2.y;
             }
@@ -477,7 +635,10 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
 #pragma unroll
             for (int j = 0; j < DPL; ++j) {
                 const int row = lane + 32 * j;
-                tod[j] = rb.tod[row][k];
+                if constexpr (TMA)
+                    tod[j] = *reinterpret_cast<const double*>(tod_tile + (row_swz ^ ((unsigned)k << 3)));
+                else
+                    tod[j] = rb.tod[row][k];
                 dflag[j] = fmask[j] & bit;
             }
             // fold the previous sample while those shared-memory loads are in flight
@@ -500,17 +661,108 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
             for (int j = 0; j < DPL; ++j)
                 load_slot<P>(sl[j], a, nxt.d0 + lane + 32 * j, lane + 32 * j < nxt.nrows, nxt.d0);
         }
-        __syncwarp();  // all lanes are done with buf[p] and st before they are refilled
+        __syncwarp();  // all lanes are done with buffer p and st before they are refilled
         cur = nxt;
         p ^= 1;
     }
-    cp_async_wait_all();
+    if constexpr (!TMA) cp_async_wait_all();
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL>
-cudaError_t launch_t(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
-    auto kern = pointing_to_map_kernel<NEST, NNZ, HWP, DEBUG, WIDE, DPL>;
-    const size_t smem = sizeof(WarpSmem<DPL>) * kWarps;
+// Tensor-map encoder from the driver, fetched through the runtime (no link against libcuda).
+PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* ptr = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &ptr, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(ptr);
+    });
+    return fn;
+}
+
+bool encode_map(CUtensorMap* m, CUtensorMapDataType type, cuuint32_t rank, const void* base, const cuuint64_t* dims,
+                const cuuint64_t* strides, const cuuint32_t* box, CUtensorMapSwizzle swz) {
+    const cuuint32_t es[2] = {1, 1};
+    return tensor_map_encoder()(m, type, rank, const_cast<void*>(base), dims, strides, box, es,
+                                CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; }
+
+const cuuint64_t kNoStrides[1] = {0};  // rank-1 maps have no strides (a non-null array is passed anyway)
+
+// The TMA path applies when every staged array is 16-byte aligned, rows of the TOD and the
+// det flags are multiples of 16 bytes (n_samp % 16 == 0) and sample / detector coordinates
+// fit the 32-bit TMA coordinates; otherwise the cp.async path runs (same results).
+thread_local const char* t_fused_path = "";
+
+bool make_tma_maps(const FusedArgs& a, TmaMaps* tm) {
+#ifdef TB_NO_TMA
+    t_fused_path = "cp.async (TMA disabled at build time)";
+    return false;
+#endif
+    if (!tensor_map_encoder()) {
+        t_fused_path = "cp.async (no cuTensorMapEncodeTiled)";
+        return false;
+    }
+    if (a.n_samp % 16 != 0 || a.n_samp >= (int64_t(1) << 31) || a.n_det >= (int64_t(1) << 31)) {
+        t_fused_path = "cp.async (n_samp % 16 != 0 or sizes beyond 32-bit TMA coordinates)";
+        return false;
+    }
+    if (!aligned16(a.det_data) || !aligned16(a.boresight) || (a.det_flags && !aligned16(a.det_flags)) ||
+        (a.hwp && !aligned16(a.hwp)) || (a.shared_flags && !aligned16(a.shared_flags))) {
+        t_fused_path = "cp.async (an input array is not 16-byte aligned)";
+        return false;
+    }
+    t_fused_path = "cp.async (tensor map encoding failed)";
+    std::memset(tm, 0, sizeof(*tm));
+    const cuuint64_t ns = (cuuint64_t)a.n_samp, nd = (cuuint64_t)a.n_det;
+    {
+        const cuuint64_t dims[2] = {ns, nd}, strides[1] = {ns * 8};
+        const cuuint32_t box[2] = {16, 32};
+        if (!encode_map(&tm->tod, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, a.det_data, dims, strides, box,
+                        CU_TENSOR_MAP_SWIZZLE_128B))
+            return false;
+    }
+    if (a.det_flags) {
+        const cuuint64_t dims[2] = {ns, nd}, strides[1] = {ns};
+        const cuuint32_t box[2] = {16, 32};
+        if (!encode_map(&tm->flg, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, a.det_flags, dims, strides, box,
+                        CU_TENSOR_MAP_SWIZZLE_NONE))
+            return false;
+    }
+    {
+        const cuuint64_t dims[2] = {4, ns}, strides[1] = {32};
+        const cuuint32_t box[2] = {4, 16};
+        if (!encode_map(&tm->bore, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, a.boresight, dims, strides, box,
+                        CU_TENSOR_MAP_SWIZZLE_NONE))
+            return false;
+    }
+    if (a.hwp) {
+        const cuuint64_t dims[1] = {ns};
+        const cuuint32_t box[1] = {16};
+        if (!encode_map(&tm->hwp, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 1, a.hwp, dims, kNoStrides, box,
+                        CU_TENSOR_MAP_SWIZZLE_NONE))
+            return false;
+    }
+    if (a.shared_flags) {
+        const cuuint64_t dims[1] = {ns};
+        const cuuint32_t box[1] = {16};
+        if (!encode_map(&tm->sflg, CU_TENSOR_MAP_DATA_TYPE_UINT8, 1, a.shared_flags, dims, kNoStrides, box,
+                        CU_TENSOR_MAP_SWIZZLE_NONE))
+            return false;
+    }
+    return true;
+}
+
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL, bool TMA>
+cudaError_t launch_k(const WorkList& wl, const FusedArgs& a, const TmaMaps& tm, unsigned long long* sched,
+                     cudaStream_t st) {
+    auto kern = pointing_to_map_kernel<NEST, NNZ, HWP, DEBUG, WIDE, DPL, TMA>;
+    const size_t smem = TMA ? sizeof(TmaWarpSmem) * kWarps + 1024 : sizeof(WarpSmem<DPL>) * kWarps;
     static int blocks_per_sm = 0;
     static std::once_flag once;
     std::call_once(once, [&] {
@@ -525,8 +777,19 @@ cudaError_t launch_t(const WorkList& wl, const FusedArgs& a, unsigned long long*
     if (grid <= 0) return cudaSuccess;
     cudaError_t e = cudaMemsetAsync(sched, 0, sizeof(unsigned long long), st);
     if (e != cudaSuccess) return e;
-    kern<<<(unsigned)grid, kWarps * 32, smem, st>>>(wl.chunks, wl.n_chunks, a, make_geom(a.nside), sched);
+    kern<<<(unsigned)grid, kWarps * 32, smem, st>>>(wl.chunks, wl.n_chunks, a, make_geom(a.nside), sched, tm);
     return cudaGetLastError();
+}
+
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL>
+cudaError_t launch_t(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
+    TmaMaps tm;
+    if (DPL == 1 && make_tma_maps(a, &tm)) {
+        t_fused_path = "tma";
+        return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, 1, true>(wl, a, tm, sched, st);
+    }
+    std::memset(&tm, 0, sizeof(tm));
+    return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, DPL, false>(wl, a, tm, sched, st);
 }
 
 template <bool NEST, int NNZ, bool HWP, bool DEBUG>
@@ -798,6 +1061,8 @@ cudaError_t launch_pointing_to_tod(const WorkList& wl, const FusedArgs& a, unsig
     if (a.nest) return a.nnz == 3 ? dispatch_scan<true, 3>(wl, a, sched, st) : dispatch_scan<true, 1>(wl, a, sched, st);
     return a.nnz == 3 ? dispatch_scan<false, 3>(wl, a, sched, st) : dispatch_scan<false, 1>(wl, a, sched, st);
 }
+
+const char* last_fused_path() { return t_fused_path; }
 
 cudaError_t launch_pointing_to_map(const WorkList& wl, const FusedArgs& a, unsigned long long* sched,
                                    cudaStream_t st) {

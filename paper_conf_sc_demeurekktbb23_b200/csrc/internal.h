@@ -88,6 +88,9 @@ cudaError_t launch_scan_map(const WorkList& wl, const MapGeom& mg, const double*
                             cudaStream_t st);
 cudaError_t launch_pointing_to_map(const WorkList& wl, const FusedArgs& a, unsigned long long* sched,
                                    cudaStream_t st);
+// How the last toast_pointing_to_map call on this host thread staged its inputs ("tma", or
+// "cp.async (<reason>)").
+const char* last_fused_path();
 cudaError_t launch_pointing_to_tod(const WorkList& wl, const FusedArgs& a, unsigned long long* sched,
                                    cudaStream_t st);
 

@@ -58,15 +58,18 @@ def main():
     nds = w.det_samples
     n_det, n_samp, ivs = w.n_det, w.n_samp, w.intervals
     dev = "cuda"
-    quats = torch.zeros((n_det, n_samp, 4), dtype=torch.float64, device=dev)
-    pix = torch.zeros((n_det, n_samp), dtype=torch.int64, device=dev)
-    wts = torch.zeros((n_det, n_samp, 3), dtype=torch.float64, device=dev)
+    only = [x for x in args.only.split(",") if x]
+    fused_only = bool(only) and all("fused" in o or "pointing_to_" in o for o in only)
+    # unfused intermediates (32 + 8 + 24 B per det-sample) only when an unfused entry is timed
+    shp = (1, 1) if fused_only else (n_det, n_samp)
+    quats = torch.zeros((*shp, 4), dtype=torch.float64, device=dev)
+    pix = torch.zeros(shp, dtype=torch.int64, device=dev)
+    wts = torch.zeros((*shp, 3), dtype=torch.float64, device=dev)
     tod2 = dw.det_data.clone()
     rng = np.random.default_rng(0)
     m = torch.from_numpy(rng.normal(size=(w.n_submap, w.n_pix_submap, 3))).to(dev)
     out = []
 
-    only = [x for x in args.only.split(",") if x]
 
     def timed_if(name, fn):
         return timed(fn, args.reps) if not only or any(o in name for o in only) else None
@@ -75,6 +78,8 @@ def main():
         if ms is None:
             return
         d = {"workload": args.workload, "entry": name, "ms": ms, "det_samples_per_s": nds / (ms / 1e3)}
+        if "pointing_to_map" in name:
+            d["staging"] = binding.last_fused_path()
         if bytes_per is not None:
             gbs = bytes_per * nds / (ms / 1e3) / 1e9
             d.update(alg_bytes_per_det_sample=bytes_per, achieved_gbs=gbs, hbm_frac=gbs / hbm)
@@ -83,9 +88,10 @@ def main():
 
     sf = dict(shared_flags=dw.shared_flags, shared_flag_mask=w.shared_flag_mask)
     # the unfused chain's intermediates, computed once untimed so any --only subset sees real data
-    binding.pointing_detector(dw.fp_quats, dw.boresight, ivs, quats, **sf)
-    binding.pixels_healpix(quats, ivs, w.nside, w.nest, w.n_pix_submap, pix, **sf)
-    binding.stokes_weights_iqu(quats, ivs, dw.epsilon, w.cal, wts, hwp=dw.hwp)
+    if not fused_only:
+        binding.pointing_detector(dw.fp_quats, dw.boresight, ivs, quats, **sf)
+        binding.pixels_healpix(quats, ivs, w.nside, w.nest, w.n_pix_submap, pix, **sf)
+        binding.stokes_weights_iqu(quats, ivs, dw.epsilon, w.cal, wts, hwp=dw.hwp)
     rep("pointing_to_map (fused A1-A4)", timed_if("pointing_to_map (fused A1-A4)", lambda: dw.pointing_to_map()))
     rep("pointing_to_tod (fused A1-A3+A5)", timed_if("pointing_to_tod (fused A1-A3+A5)", lambda: binding.pointing_to_tod(dw.fp_quats, dw.boresight, dw.epsilon, w.cal, ivs, w.nside, w.nest, 3,
                                               dw.global2local, w.n_pix_submap, m, tod2, hwp=dw.hwp, **sf)), 16)

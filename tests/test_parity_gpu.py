@@ -72,6 +72,8 @@ FUSED_CASES = {
     "c4_sat_nest_2048": dict(name="c4", n_det=36, n_samp=40_000),
     "c5_nest_4096": dict(name="c5", n_det=24, n_samp=133_200),
     "c1_ring_nest_swap": dict(name="c1", n_samp=50_000, nest=True, nside=128),
+    # n_samp % 16 != 0: the cp.async staging path instead of the TMA path
+    "c2_cp_async_path": dict(name="c2", n_det=40, n_samp=100_003),
 }
 
 
@@ -109,6 +111,28 @@ def test_fused_pointing_to_map(case):
     torch.cuda.synchronize()
     check_map(dw.zmap.cpu().numpy(), zo_r, abs_r)
     np.testing.assert_array_equal(dw.hit_submaps.cpu().numpy(), hits_expect)
+
+
+def test_fused_tma_and_cp_async_paths():
+    """The same workload staged by TMA (aligned TOD) and by cp.async (TOD base only 8-byte
+    aligned, so the TMA constraints fail) gives the oracle's map either way."""
+    w = synth.make_workload("c2", n_det=36, n_samp=64_000)
+    zo, absmap, ho, po, wo = _oracle_fused(w)
+    buf = torch.empty(w.n_det * w.n_samp + 1, dtype=torch.float64, device=DEV)
+    odd = buf[1:].view(w.n_det, w.n_samp)
+    odd.copy_(torch.from_numpy(np.ascontiguousarray(w.det_data)))
+    assert odd.data_ptr() % 16 == 8
+    for det_data, path in ((None, "tma"), (odd, "cp.async")):
+        dw = DeviceWorkload.upload(w, DEV, det_data=det_data)
+        pix_g = torch.full((w.n_det, w.n_samp), -7, dtype=torch.int64, device=DEV)
+        dw.pointing_to_map(pixels_out=pix_g)
+        torch.cuda.synchronize()
+        assert binding.last_fused_path().startswith(path), binding.last_fused_path()
+        pg = pix_g.cpu().numpy()
+        n_in = int(_in_mask(w.intervals, 1, w.n_samp).sum()) * w.n_det
+        mism = classify_pixel_mismatches(pg, po, _probe(w), w.nside, w.nest, n_in)
+        zo_r, abs_r = reconcile_map(zo.copy(), absmap.copy(), mism, pg, po, wo, w, w.global2local, w.n_pix_submap)
+        check_map(dw.zmap.cpu().numpy(), zo_r, abs_r)
 
 
 def test_fused_integer_inputs_give_exact_hit_counts():
@@ -159,10 +183,14 @@ def test_fused_extreme_nside(nside, nest):
     check_map(dw.zmap.cpu().numpy(), zo_r, abs_r)
 
 
-def test_fused_edge_intervals():
-    """Empty interval list, single-sample intervals, chunk-boundary lengths (255/256/257)."""
-    w = synth.make_workload("c1", n_samp=5000)
-    for ivs in ([], [(0, 0)], [(0, 254), (300, 555), (600, 856), (4999, 4999)], [(10, 10), (11, 11), (12, 4000)]):
+@pytest.mark.parametrize("n_samp", [5000, 5008])  # cp.async path (n_samp % 16 != 0) and TMA path
+def test_fused_edge_intervals(n_samp):
+    """Empty interval list, single-sample intervals, chunk-boundary lengths (255/256/257),
+    odd first samples (the TMA box then starts one sample earlier), the last sample."""
+    w = synth.make_workload("c1", n_samp=n_samp)
+    last = n_samp - 1
+    for ivs in ([], [(0, 0)], [(0, 254), (300, 555), (600, 856), (last, last)], [(10, 10), (11, 11), (12, 4000)],
+                [(1, 1), (3, 17), (33, 160), (161, 290), (4001, last)], [(last - 16, last)]):
         w.intervals = ivs
         zo, absmap, ho, po, wo = _oracle_fused(w)
         dw = DeviceWorkload.upload(w, DEV)
