@@ -42,10 +42,11 @@ constexpr double kTanPi8 = 0.41421356237309504880;
 // Constants whose low word is non-zero are kept in the constant bank so that the fp64
 // instructions take them as c[][] operands: written as literals, the compiler re-materialises
 // them with two UMOVs per use inside the hot loop once the uniform registers run out.
-static __constant__ double kC[3] = {kTanPi8, 1e-100, 2.0 / 3.0};
+static __constant__ double kC[4] = {kTanPi8, 1e-100, 2.0 / 3.0, 0.99};
 #define TB_TAN_PI8 (::toastb200::kC[0])
 #define TB_TINY (::toastb200::kC[1])
 #define TB_TWO_THIRD (::toastb200::kC[2])
+#define TB_CAP_SINTHETA_Z (::toastb200::kC[3])
 
 // 1/x for finite x > 0 (no IEEE rounding guarantee; <= ~1 ulp): MUFU seed + 2 Newton steps.
 __device__ __forceinline__ double fast_rcp(double x) {
@@ -161,23 +162,36 @@ __device__ __forceinline__ double fast_sqrt(double x) {
 // reduction by pi/2 with the fdlibm split constants, then the fdlibm __kernel_sin/__kernel_cos
 // minimax polynomials on [-pi/4, pi/4].  Max error 2.2e-16 (checked against libm over [0, 8 pi));
 // branch-free, no local-memory Payne-Hanek path (unlike the generic sincos()).
+// (reduction constants and polynomial coefficients in the constant bank: c[][] operands
+// instead of two UMOVs per literal)
+static __constant__ double kSinCos[15] = {
+    0.63661977236758134308,      // 2/pi
+    1.57079632673412561417e+00,  // pi/2, high part
+    6.07710050650619224932e-11,  // pi/2, low part
+    1.58969099521155010221e-10,  -2.50507602534068634195e-08, 2.75573137070700676789e-06,
+    -1.98412698298579493134e-04, 8.33333333332248946124e-03,  -1.66666666666666324348e-01,
+    -1.13596475577881948265e-11, 2.08757232129817482790e-09,  -2.75573143513906633035e-07,
+    2.48015872894767294178e-05,  -1.38888888888741095749e-03, 4.16666666666666019037e-02,
+};
+
 __device__ __forceinline__ void small_sincos(double a, double* sp, double* cp) {
-    const double k = rint(a * 0.63661977236758134308);
-    const double r = fma(-k, 6.07710050650619224932e-11, fma(-k, 1.57079632673412561417e+00, a));
+    const double* C = kSinCos;
+    const double k = rint(a * C[0]);
+    const double r = fma(-k, C[2], fma(-k, C[1], a));
     const double z = r * r;
-    double ps = 1.58969099521155010221e-10;
-    ps = fma(ps, z, -2.50507602534068634195e-08);
-    ps = fma(ps, z, 2.75573137070700676789e-06);
-    ps = fma(ps, z, -1.98412698298579493134e-04);
-    ps = fma(ps, z, 8.33333333332248946124e-03);
-    ps = fma(ps, z, -1.66666666666666324348e-01);
+    double ps = C[3];
+    ps = fma(ps, z, C[4]);
+    ps = fma(ps, z, C[5]);
+    ps = fma(ps, z, C[6]);
+    ps = fma(ps, z, C[7]);
+    ps = fma(ps, z, C[8]);
     const double sn = fma(r * z, ps, r);
-    double pc = -1.13596475577881948265e-11;
-    pc = fma(pc, z, 2.08757232129817482790e-09);
-    pc = fma(pc, z, -2.75573143513906633035e-07);
-    pc = fma(pc, z, 2.48015872894767294178e-05);
-    pc = fma(pc, z, -1.38888888888741095749e-03);
-    pc = fma(pc, z, 4.16666666666666019037e-02);
+    double pc = C[9];
+    pc = fma(pc, z, C[10]);
+    pc = fma(pc, z, C[11]);
+    pc = fma(pc, z, C[12]);
+    pc = fma(pc, z, C[13]);
+    pc = fma(pc, z, C[14]);
     const double cs = fma(z * z, pc, fma(-0.5, z, 1.0));
     const int q = (int)k & 3;
     const double s0 = (q & 1) ? cs : sn;
@@ -291,7 +305,7 @@ __device__ __forceinline__ int64_t loc2pix(const HealpixGeom& g, double dz, doub
     }
     // polar caps; the well-conditioned sin(theta) form for za >= 0.99 (reading S5)
     double tmp;
-    if (za < 0.99) {
+    if (za < TB_CAP_SINTHETA_Z) {
         tmp = __dmul_rn(g.dnside, __dsqrt_rn(__dmul_rn(3.0, __dsub_rn(1.0, za))));
     } else {
         const double sth = __dsqrt_rn(__dadd_rn(__dmul_rn(dx, dx), __dmul_rn(dy, dy)));
@@ -363,7 +377,7 @@ __device__ __forceinline__ int loc2pix32(const HealpixGeom& g, double dz, double
         }
     }
     double tmp;
-    if (za < 0.99) {
+    if (za < TB_CAP_SINTHETA_Z) {
         tmp = __dmul_rn(g.dnside, fast_sqrt(__dmul_rn(3.0, __dsub_rn(1.0, za))));
     } else {
         const double sth = __dsqrt_rn(__dadd_rn(__dmul_rn(dx, dx), __dmul_rn(dy, dy)));

@@ -432,8 +432,10 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
     const int wid = threadIdx.x >> 5;
     // cp.async path: WarpSmem<DPL>; TMA path: TmaWarpSmem (1 KB-aligned, see launch_t)
     WarpSmem<DPL>& sm = reinterpret_cast<WarpSmem<DPL>*>(smem_raw)[wid];
-    TmaWarpSmem& tw = reinterpret_cast<TmaWarpSmem*>(
-        (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023))[wid];
+    // (offset arithmetic on the __shared__ array itself, so every access below stays an LDS;
+    // the alignment that matters for TMA and the swizzle is that of the shared-window offset)
+    const unsigned pad1k = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
+    TmaWarpSmem& tw = reinterpret_cast<TmaWarpSmem*>(smem_raw + pad1k)[wid];
     constexpr int kRows = 32 * DPL;
     const int64_t n_groups = (a.n_det + kRows - 1) / kRows;
     const int64_t n_items = n_chunks * n_groups;
@@ -548,6 +550,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
             __syncwarp();
         }
         if (nxt.item >= 0) issue(p ^ 1, nxt);
+        __syncwarp();  // reconverge after the lane-0 / spin-wait paths (else the state code below runs twice)
 
         RawBlock<DPL>& rb = sm.buf[p];
         // per-sample state (lanes 0..15); bit k of pmask = sample k is pixelised
