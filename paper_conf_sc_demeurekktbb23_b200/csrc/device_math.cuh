@@ -48,13 +48,15 @@ static __constant__ double kC[4] = {kTanPi8, 1e-100, 2.0 / 3.0, 0.99};
 #define TB_TWO_THIRD (::toastb200::kC[2])
 #define TB_CAP_SINTHETA_Z (::toastb200::kC[3])
 
-// 1/x for finite x > 0 (no IEEE rounding guarantee; <= ~1 ulp): MUFU seed + 2 Newton steps.
+// 1/x for finite x > 0 (no IEEE rounding guarantee; <= ~1 ulp): MUFU seed + ONE cubic step,
+// r' = r + r (e + e^2) with e = 1 - x r.  Measured on B200 (scripts/mufu_precision.cu, 2^24
+// inputs): the seed's relative error is <= 2^-19.9, after the cubic step <= 2^-52.0 (1 ulp);
+// 3 DFMA instead of the 4 of two quadratic steps.
 __device__ __forceinline__ double fast_rcp(double x) {
     double r;
     asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(x));
-    r = fma(r, fma(-x, r, 1.0), r);
-    r = fma(r, fma(-x, r, 1.0), r);
-    return r;
+    const double e = fma(-x, r, 1.0);
+    return fma(r, fma(e, e, e), r);
 }
 
 // tt = fmodulo(2 atan2(y, x) / pi, 4) in [0, 4) -- the HEALPix longitude in quarter turns --
@@ -77,7 +79,9 @@ struct QtPrep {
 };
 
 __device__ __forceinline__ QtPrep qt_prepare(double x, double y) {
-    const double ax = fabs(x), ay = fabs(y);
+    // |x| + 1e-100: the guard that makes x = y = 0 give t = 0 (den >= 1e-100) costs nothing —
+    // the DADD replaces the one that materialises |x| — and changes nothing for |x| > 1e-84.
+    const double ax = fabs(x) + TB_TINY, ay = fabs(y);
     const bool swap = ay > ax;
     const double mx = swap ? ay : ax;
     const double mn = swap ? ax : ay;
@@ -85,11 +89,12 @@ __device__ __forceinline__ QtPrep qt_prepare(double x, double y) {
     const double beta = big ? 1.0 : 0.0;
     QtPrep q;
     q.num = fma(-beta, mx, mn);
-    q.den = fma(beta, mn, mx) + TB_TINY;  // x = y = 0 -> t = 0; changes nothing for den > 1e-84
-    // K in units of half a quarter turn; S = (-1)^(swap + x<0 + y<0)
+    q.den = fma(beta, mn, mx);
+    // K in units of half a quarter turn; S = (-1)^(swap + x<0 + y<0).  The signs are the sign
+    // BITS (integer tests, not fp64 compares), which is also C99 atan2's treatment of -0.
     int kk = big ? 1 : 0;
     kk = swap ? 2 - kk : kk;
-    const bool xneg = x < 0.0, yneg = y < 0.0;
+    const bool xneg = __double2hiint(x) < 0, yneg = __double2hiint(y) < 0;
     kk = xneg ? 4 - kk : kk;
     q.kk = yneg ? 8 - kk : kk;
     q.neg = swap ^ xneg ^ yneg;
@@ -122,7 +127,7 @@ __device__ __forceinline__ double qt_finish(const QtPrep& q, double t) {
     const double st = __hiloint2double(__double2hiint(t) ^ (q.neg ? (int)0x80000000 : 0), __double2loint(t));
     const double half_k = __hiloint2double(0x43200000, q.kk) - 2251799813685248.0;
     double tt = fma(st, p, half_k);
-    if (tt >= 4.0) tt = 0.0;
+    if (__double2hiint(tt) >= 0x40100000) tt = 0.0;  // tt >= 4 (tt >= -0 here): an integer compare
     return tt;
 }
 
@@ -147,12 +152,13 @@ __device__ __forceinline__ int floor_nonneg(double x) {
 }
 
 // sqrt(x) for x >= 0.03 (the HEALPix cap term 3(1 - |z|) with |z| < 0.99): reciprocal square
-// root seed + two Newton steps, within ~1 ulp (not IEEE-rounded; only floors of it matter, and
-// those may differ from the oracle only within ~1e-15 rad of a pixel boundary).
+// root seed (relative error <= 2^-20.0 measured, scripts/mufu_precision.cu), one Newton step on
+// 1/sqrt (<= 2^-39.5 measured), then one Newton step on sqrt itself, which squares the error
+// again: within ~1 ulp (not IEEE-rounded; only floors of it matter, and those may differ from
+// the oracle only within ~1e-15 rad of a pixel boundary).
 __device__ __forceinline__ double fast_sqrt(double x) {
     double y;
     asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(x));
-    y = y * fma(-0.5 * x, y * y, 1.5);
     y = y * fma(-0.5 * x, y * y, 1.5);
     const double r = x * y;
     return fma(0.5 * y, fma(-r, r, x), r);  // one Newton step on sqrt itself
@@ -409,6 +415,78 @@ __device__ __forceinline__ int loc2pix32(const HealpixGeom& g, double dz, double
     }
 }
 
+// Run key of the pixel (fused kernels): RING -> the pixel; NEST -> face*N^2 + iy*N + ix, a
+// packing that costs two IMADs per det-sample instead of the bit interleave, which
+// key_to_pix32 applies once per run.  Same floors, in the same order and rounding, as
+// loc2pix32.
+template <bool NEST>
+__device__ __forceinline__ int loc2key32(const HealpixGeom& g, double dz, double tt, double dx, double dy) {
+    const double za = fabs(dz);
+    const int nside = (int)g.nside;
+    const int m = nside - 1;
+    if (za <= TB_TWO_THIRD) {
+        const double temp1 = __dmul_rn(g.dnside, __dadd_rn(0.5, tt));
+        const double temp2 = __dmul_rn(__dmul_rn(g.dnside, dz), 0.75);
+        const int jp = floor_nonneg(__dsub_rn(temp1, temp2));
+        const int jm = floor_nonneg(__dadd_rn(temp1, temp2));
+        if (!NEST) {
+            const int nl4 = 4 * nside;
+            const int ir = nside + 1 + jp - jm;
+            const int kshift = 1 - (ir & 1);
+            const int t1 = jp + jm - nside + kshift + 1 + 2 * nl4;
+            const int ip = (t1 >> 1) & (nl4 - 1);
+            return (int)g.ncap + nl4 * (ir - 1) + ip;
+        } else {
+            const int ifp = jp >> g.order;
+            const int ifm = jm >> g.order;
+            const int face = (ifp == ifm) ? (ifp | 4) : ((ifp < ifm) ? ifp : (ifm + 8));
+            const int ix = jm & m;
+            const int iy = (jp & m) ^ m;  // nside - 1 - (jp & (nside - 1))
+            return (face * nside + iy) * nside + ix;
+        }
+    }
+    double tmp;
+    if (za < TB_CAP_SINTHETA_Z) {
+        tmp = __dmul_rn(g.dnside, fast_sqrt(__dmul_rn(3.0, __dsub_rn(1.0, za))));
+    } else {
+        const double sth = __dsqrt_rn(__dadd_rn(__dmul_rn(dx, dx), __dmul_rn(dy, dy)));
+        tmp = __ddiv_rn(__dmul_rn(g.dnside, sth), __dsqrt_rn(__ddiv_rn(__dadd_rn(1.0, za), 3.0)));
+    }
+    if (!NEST) {
+        const double tp = __dsub_rn(tt, small_int_to_double(floor_nonneg(tt)));
+        const int jp = floor_nonneg(__dmul_rn(tp, tmp));
+        const int jm = floor_nonneg(__dmul_rn(__dsub_rn(1.0, tp), tmp));
+        const int ir = jp + jm + 1;
+        int ip = floor_nonneg(__dmul_rn(tt, small_int_to_double(ir)));
+        if (ip >= 4 * ir) ip -= 4 * ir;
+        return (dz > 0.0) ? 2 * ir * (ir - 1) + ip : (int)g.npix - 2 * ir * (ir + 1) + ip;
+    } else {
+        int ntt = floor_nonneg(tt);
+        if (ntt > 3) ntt = 3;
+        const double tp = __dsub_rn(tt, small_int_to_double(ntt));
+        int jp = floor_nonneg(__dmul_rn(tp, tmp));
+        int jm = floor_nonneg(__dmul_rn(__dsub_rn(1.0, tp), tmp));
+        if (jp > m) jp = m;
+        if (jm > m) jm = m;
+        int face, ix, iy;
+        if (dz >= 0.0) {
+            face = ntt; ix = m - jm; iy = m - jp;
+        } else {
+            face = ntt + 8; ix = jp; iy = jm;
+        }
+        return (face * nside + iy) * nside + ix;
+    }
+}
+
+// Pixel of a run key (see loc2key32).
+template <bool NEST>
+__device__ __forceinline__ int key_to_pix32(int key, const HealpixGeom& g) {
+    if (!NEST) return key;
+    const int m = (int)g.nside - 1;
+    const int face_bits = key & ~((1 << (2 * g.order)) - 1);  // face * nside^2
+    return face_bits | (int)interleave16((uint32_t)(key & m), (uint32_t)((key >> g.order) & m));
+}
+
 // tt = fmodulo(phi * 2/pi, 4) in [0, 4) with phi = atan2(dy, dx) (phi := 0 at dx = dy = 0, S3).
 __device__ __forceinline__ double phi_to_tt(double dx, double dy) { return quarter_turns(dx, dy); }
 
@@ -426,6 +504,22 @@ __device__ __forceinline__ void cos_sin_2psi(double bx, double by, double& c2, d
     const double inv = fast_rcp(r);
     c2 = fma(-by, by, bx2 + 1e-100) * inv;
     s2 = 2.0 * bx * by * inv;
+}
+
+// Longitude in quarter turns, and the pieces of the polarisation weights, with ONE reciprocal:
+// returns tt; sets A = r cos 2psi, B = r sin 2psi (r = bx^2 + by^2 + 1e-100, so (bx, by) = 0
+// gives (1, 0), reading S10) and invr = 1/r.  1/(den r) gives 1/den = r/(den r) and
+// 1/r = den/(den r).
+__device__ __forceinline__ double lon_pol_raw(double dx, double dy, double bx, double by, double& A, double& B,
+                                              double& invr) {
+    const QtPrep q = qt_prepare(dx, dy);
+    const double bx2 = fma(bx, bx, TB_TINY);
+    const double r = fma(by, by, bx2);
+    const double inv = fast_rcp(q.den * r);
+    invr = q.den * inv;
+    A = fma(-by, by, bx2);
+    B = (bx + bx) * by;
+    return qt_finish(q, q.num * (r * inv));
 }
 
 // Longitude in quarter turns AND (cos 2psi, sin 2psi) with ONE reciprocal: 1/(den r) gives

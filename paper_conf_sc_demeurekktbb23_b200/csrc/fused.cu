@@ -208,13 +208,36 @@ __device__ __forceinline__ int64_t submap_of(P pix, const MapGeom& mg) {
     return mg.sm_shift >= 0 ? (int64_t)(pix >> mg.sm_shift) : (int64_t)pix / mg.n_pix_submap;
 }
 
+// Pixel of a run key: 32-bit NEST keys are the cheap (face, iy, ix) packing of loc2key32;
+// 64-bit keys (nside > 8192) and RING keys are the pixel itself.
+template <bool NEST, bool WIDE>
+__device__ __forceinline__ typename PixT<WIDE>::T key_to_pix(typename PixT<WIDE>::T key, const HealpixGeom& g) {
+    if constexpr (WIDE) {
+        return key;
+    } else {
+        return key_to_pix32<NEST>(key, g);
+    }
+}
+
 // A run starts: mark its submap hit (as A2 does) and issue the global2local lookup now, so
 // the load latency is hidden behind the run's samples instead of stalling the flush.  The hit
 // flag is stored only when the lane's submap CHANGES: thousands of warps re-writing the same
-// few bytes of hit_submaps serialise in L2 and cost as much as the whole computation.
-template <typename P>
-__device__ __forceinline__ int64_t start_run(P pix, const FusedArgs& a, int64_t& last_sm) {
-    const int64_t sm = submap_of<P>(pix, a.map);
+// few bytes of hit_submaps serialise in L2 and cost as much as the whole computation.  `lp`
+// receives the pixel's index inside its submap.
+template <bool NEST, bool WIDE>
+__device__ __forceinline__ int64_t start_run(typename PixT<WIDE>::T key, const FusedArgs& a, const HealpixGeom& g,
+                                             typename PixT<WIDE>::T& last_sm, typename PixT<WIDE>::T& lp) {
+    using P = typename PixT<WIDE>::T;
+    const MapGeom& mg = a.map;
+    const P pix = key_to_pix<NEST, WIDE>(key, g);
+    P sm;
+    if (mg.sm_shift >= 0) {
+        sm = pix >> mg.sm_shift;
+        lp = pix & (P)(mg.n_pix_submap - 1);
+    } else {
+        sm = pix / (P)mg.n_pix_submap;
+        lp = pix - sm * (P)mg.n_pix_submap;
+    }
 #ifndef TB_X_NOHIT
     if (a.hit_submaps && sm != last_sm) {
         a.hit_submaps[sm] = 1;
@@ -224,18 +247,24 @@ __device__ __forceinline__ int64_t start_run(P pix, const FusedArgs& a, int64_t&
 #ifdef TB_X_NOG2L
     return sm;
 #else
-    return __ldg(&a.map.global2local[sm]);
+    return __ldg(&mg.global2local[sm]);
 #endif
 }
 
-// A run ends: one fp64 red per Stokes component (nothing if the submap has no storage).
-template <int NNZ, typename P>
-__device__ __forceinline__ void flush(P pix, int64_t loc, double a0, double a1, double a2, const FusedArgs& a) {
+// A run ends: one fp64 red per Stokes component (nothing if the submap has no storage).  Up to
+// nside 8192 the map element index fits 32 bits (< 12 * 8192^2 pixels), so the address is one
+// IMAD + one IMAD.WIDE.U32.
+template <int NNZ, bool WIDE>
+__device__ __forceinline__ void flush(int64_t loc, typename PixT<WIDE>::T lp, double a0, double a1, double a2,
+                                      const FusedArgs& a) {
     if (loc < 0) return;
-    const MapGeom& mg = a.map;
-    const int64_t lp = mg.sm_shift >= 0 ? (int64_t)(pix & (P)(mg.n_pix_submap - 1))
-                                        : (int64_t)pix - submap_of<P>(pix, mg) * mg.n_pix_submap;
-    double* dst = a.zmap + (loc * mg.n_pix_submap + lp) * NNZ;
+    double* dst;
+    if constexpr (WIDE) {
+        dst = a.zmap + (loc * a.map.n_pix_submap + lp) * NNZ;
+    } else {
+        const unsigned idx = (unsigned)loc * (unsigned)a.map.n_pix_submap + (unsigned)lp;
+        dst = a.zmap + (size_t)idx * NNZ;
+    }
     atomicAdd(dst, a0);
     if (NNZ == 3) {
         atomicAdd(dst + 1, a1);
@@ -249,11 +278,12 @@ struct Slot {
     double s_cal;   // det_scale * cal       (I weight folded into the noise weight)
     double s_eta;   // det_scale * eta * cal (Q/U amplitude folded into the noise weight)
     double etacal;  // debug outputs only
-    P run_pix;
+    P run_key;            // key of the run being aggregated (-1: none)
+    P run_lp;             // its pixel's index inside the submap
     int64_t run_loc;      // global2local of the run's submap, LOADED WHEN THE RUN STARTS
-    int64_t last_sm;      // last submap this lane marked in hit_submaps
+    P last_sm;            // last submap this lane marked in hit_submaps
     double r0, r1, r2;
-    P pend_pix;           // pending (not yet aggregated) det-sample
+    P pend_key;           // pending (not yet aggregated) det-sample
     double p0, p1, p2;
     bool ok;
 };
@@ -274,96 +304,99 @@ __device__ __forceinline__ void load_slot(Slot<P>& sl, const FusedArgs& a, int64
     // a lane without a detector contributes exactly 0 (aggregate() adds unconditionally)
     sl.s_cal = ok ? scale * a.cal : 0.0;
     sl.s_eta = ok ? scale * sl.etacal : 0.0;
-    sl.run_pix = -1;
+    sl.run_key = -1;
+    sl.run_lp = 0;
     sl.run_loc = -1;
     sl.last_sm = -1;
     sl.r0 = sl.r1 = sl.r2 = 0.0;
-    sl.pend_pix = -1;
+    sl.pend_key = -1;
     sl.p0 = sl.p1 = sl.p2 = 0.0;
     sl.ok = ok;
 }
 
-// One det-sample of slot `sl` with the per-sample state x.
+// One det-sample of slot `sl` with the per-sample state x.  `tod` is already 0 for det-flagged
+// samples (and, with debug outputs, shared-flagged ones): the block prologue zeroes them in the
+// staged tile, so no per-sample flag test is needed here.
 template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE>
 __device__ __forceinline__ void det_sample(Slot<typename PixT<WIDE>::T>& sl, const double* x, bool pixelise,
-                                           double tod, bool dflag, const HealpixGeom& g, const FusedArgs& a,
-                                           int64_t d, int64_t s) {
+                                           double tod, const HealpixGeom& g, const FusedArgs& a, int64_t d,
+                                           int64_t s) {
     using P = typename PixT<WIDE>::T;
     const double dx = x[0] * sl.u0 + x[1] * sl.u1 + x[2] * sl.u2;
     const double dy = x[3] * sl.u0 + x[4] * sl.u1 + x[5] * sl.u2;
     const double dz = x[6] * sl.u0 + x[7] * sl.u1 + x[8] * sl.u2;
     // The weight chain and the longitude chain are independent and branch-free: they are
     // written into one basic block so the scheduler can interleave them (latency-bound code).
-    // (cos 2(psi + 2 chi), sin 2(psi + 2 chi)): the Q/U weights divided by eta*cal
-    double c2 = 0.0, s2 = 0.0, tt;
+    double cw = 0.0, sw = 0.0, invr = 0.0, tt;  // r cos 2(psi + 2 chi), r sin 2(psi + 2 chi), 1/r
     if (NNZ == 3) {
         const double bx = x[6] * sl.v0 + x[7] * sl.v1 + x[8] * sl.v2;
         const double by = -(x[6] * sl.w0 + x[7] * sl.w1 + x[8] * sl.w2);
 #ifdef TB_X_NOATAN
-        tt = fabs(dx) * 3.9; c2 = bx; s2 = by;  // ablation: no longitude/weights arithmetic
+        tt = fabs(dx) * 3.9; cw = bx; sw = by; invr = 1.0;  // ablation: no longitude/weights arithmetic
 #else
-        tt = lon_pol(dx, dy, bx, by, c2, s2);  // one shared reciprocal
+        tt = lon_pol_raw(dx, dy, bx, by, cw, sw, invr);  // one shared reciprocal
 #endif
         if (HWP) {
             const double c4 = x[9], s4 = x[10];
-            const double cq = c2 * c4 - s2 * s4;
-            const double sq = s2 * c4 + c2 * s4;
-            c2 = cq;
-            s2 = sq;
+            const double cq = cw * c4 - sw * s4;
+            const double sq = sw * c4 + cw * s4;
+            cw = cq;
+            sw = sq;
         }
     } else {
         tt = quarter_turns(dx, dy);
     }
-    P pix = -1;
+    P key = -1;
     if (pixelise) {
-        if (WIDE)
-            pix = (P)loc2pix<NEST, int64_t>(g, dz, tt, dx, dy);
+        if constexpr (WIDE)
+            key = (P)loc2pix<NEST, int64_t>(g, dz, tt, dx, dy);
         else
 #ifdef TB_X_NOPIX
-            pix = (P)((int)(tt * 1000.0) & 0xffff);  // ablation: no HEALPix integer/floor logic
+            key = (P)((int)(tt * 1000.0) & 0xffff);  // ablation: no HEALPix integer/floor logic
 #else
-            pix = (P)loc2pix32<NEST>(g, dz, tt, dx, dy);
+            key = (P)loc2key32<NEST>(g, dz, tt, dx, dy);
 #endif
     }
-    if (!sl.ok) pix = -1;
+    if (!sl.ok) key = -1;
     if (DEBUG && sl.ok) {
         const int64_t o = d * a.n_samp + s;
-        if (a.pixels_out) a.pixels_out[o] = (int64_t)pix;
+        if (a.pixels_out) a.pixels_out[o] = key < 0 ? (int64_t)-1 : (int64_t)key_to_pix<NEST, WIDE>(key, g);
         if (a.weights_out) {
             a.weights_out[o * NNZ] = a.cal;
             if (NNZ == 3) {
-                a.weights_out[o * NNZ + 1] = sl.etacal * c2;
-                a.weights_out[o * NNZ + 2] = sl.etacal * s2;
+                a.weights_out[o * NNZ + 1] = sl.etacal * (cw * invr);
+                a.weights_out[o * NNZ + 2] = sl.etacal * (sw * invr);
             }
         }
     }
     // A4 contribution of this det-sample; it is folded into the lane's run by aggregate()
     // one sample LATER, so that work overlaps the shared-memory loads of the next sample.
-    // Det-flagged samples keep their pixel (they mark hit submaps, as A2 does) but add 0;
-    // so does every sample without a pixel (aggregate() adds unconditionally).
-    sl.pend_pix = pix;
-    const double tz = (dflag || (DEBUG && !pixelise)) ? 0.0 : tod;
-    sl.p0 = tz * sl.s_cal;
+    // Det-flagged samples keep their key (they mark hit submaps, as A2 does) but add 0 (their
+    // staged tod is 0); so does every sample without a key (aggregate() adds unconditionally).
+    sl.pend_key = key;
+    sl.p0 = tod * sl.s_cal;
     if (NNZ == 3) {
-        const double t = tz * sl.s_eta;
-        sl.p1 = t * c2;
-        sl.p2 = t * s2;
+        const double t = (tod * sl.s_eta) * invr;
+        sl.p1 = t * cw;
+        sl.p2 = t * sw;
     }
 }
 
 // Fold the pending contribution into the run (run-length aggregation along time).  Lanes
-// without a pixel (no detector / flagged sample) have pend_pix = -1 and never start a run.
+// without a pixel (no detector / flagged sample) have pend_key = -1 and never start a run.
 // A pending sample without a pixel carries zero contributions, so the add is unconditional
-// (one branch less per det-sample); pend_pix is not reset here because det_sample() always
-// overwrites it right after (the end-of-item call is followed by the final flush).
-template <int NNZ, typename P>
-__device__ __forceinline__ void aggregate(Slot<P>& sl, const FusedArgs& a) {
-    if (sl.pend_pix >= 0 && sl.pend_pix != sl.run_pix) {
+// (one branch less per det-sample); pend_key is not reset here because det_sample() always
+// overwrites it right after (the end-of-item call is followed by the final flush).  The first
+// run of an item flushes nothing: run_loc starts at -1.
+template <bool NEST, int NNZ, bool WIDE>
+__device__ __forceinline__ void aggregate(Slot<typename PixT<WIDE>::T>& sl, const FusedArgs& a,
+                                          const HealpixGeom& g) {
+    if (sl.pend_key >= 0 && sl.pend_key != sl.run_key) {
 #ifndef TB_X_NOFLUSH
-        if (sl.run_pix >= 0) flush<NNZ, P>(sl.run_pix, sl.run_loc, sl.r0, sl.r1, sl.r2, a);
+        flush<NNZ, WIDE>(sl.run_loc, sl.run_lp, sl.r0, sl.r1, sl.r2, a);
 #endif
-        sl.run_pix = sl.pend_pix;
-        sl.run_loc = start_run<P>(sl.pend_pix, a, sl.last_sm);
+        sl.run_key = sl.pend_key;
+        sl.run_loc = start_run<NEST, WIDE>(sl.pend_key, a, g, sl.last_sm, sl.run_lp);
         sl.r0 = sl.r1 = sl.r2 = 0.0;
     }
     sl.r0 += sl.p0;
@@ -372,7 +405,6 @@ __device__ __forceinline__ void aggregate(Slot<P>& sl, const FusedArgs& a) {
         sl.r2 += sl.p2;
     }
 }
-
 // A block of the stream: samples [s0, s0 + nb) of chunk c for detector rows d0 .. d0+nrows-1.
 struct Blk {
     int64_t item;  // < 0: end of stream
@@ -553,74 +585,92 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
         __syncwarp();  // reconverge after the lane-0 / spin-wait paths (else the state code below runs twice)
 
         RawBlock<DPL>& rb = sm.buf[p];
-        // per-sample state (lanes 0..15); bit k of pmask = sample k is pixelised
+        // Per-sample state, split over the warp: lanes 0..kBlk-1 build the boresight rotation
+        // matrix of sample `lane` (identity if shared-flagged, S2), lanes 16..16+kBlk-1 the HWP
+        // cos/sin(4 chi) of sample `lane - 16`.  Bit k of pmask = sample k is pixelised.
+        double* st_base = TMA ? &tw.st[0][0] : &sm.st[0].v[0];
         bool pixelise_me = false;
-        if (lane < kBlk) {
-            double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 1.0;
-            double c4 = 1.0, s4 = 0.0;
-            if (lane >= cur.k0 && lane < cur.k0 + cur.nb) {
-                bool flagged;
-                if constexpr (TMA) {
-                    flagged = have_sflags && (tw.sf[p].f[lane] & smask);
-                } else {
-                    const int soff =
-                        have_sflags ? (int)(reinterpret_cast<uintptr_t>(a.shared_flags + cur.s0) & 3) : 0;
-                    flagged = have_sflags && (rb.sflg[soff + lane] & smask);
+        {
+            const int ks = lane & 15;
+            const bool in_blk = ks < kBlk && ks >= cur.k0 && ks < cur.k0 + cur.nb;
+            if (lane < kBlk) {
+                double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 1.0;
+                if (in_blk) {
+                    bool flagged;
+                    if constexpr (TMA) {
+                        flagged = have_sflags && (tw.sf[p].f[lane] & smask);
+                    } else {
+                        const int soff =
+                            have_sflags ? (int)(reinterpret_cast<uintptr_t>(a.shared_flags + cur.s0) & 3) : 0;
+                        flagged = have_sflags && (rb.sflg[soff + lane] & smask);
+                    }
+                    pixelise_me = !flagged;
+                    const double* bq = TMA ? tw.bore[p][lane] : rb.bore[lane];
+                    if (!flagged) {
+                        q0 = bq[0]; q1 = bq[1]; q2 = bq[2]; q3 = bq[3];
+                    }
                 }
-                pixelise_me = !flagged;
-                const double* bq = TMA ? tw.bore[p][lane] : rb.bore[lane];
-                if (!flagged) {
-                    q0 = bq[0]; q1 = bq[1]; q2 = bq[2]; q3 = bq[3];
-                }
-                if (HWP && NNZ == 3) small_sincos(4.0 * (TMA ? tw.hwp[p][lane] : rb.hwp[lane]), &s4, &c4);
+                double m[10];
+                quat_to_matrix(q0, q1, q2, q3, m);
+                m[9] = 1.0;
+                double2* dst = reinterpret_cast<double2*>(st_base + 12 * lane);
+#pragma unroll
+                for (int i = 0; i < 4; ++i) dst[i] = make_double2(m[2 * i], m[2 * i + 1]);
+                st_base[12 * lane + 8] = m[8];
+            } else if (HWP && NNZ == 3 && ks < kBlk) {
+                double c4 = 1.0, s4 = 0.0;
+                if (in_blk) small_sincos(4.0 * (TMA ? tw.hwp[p][ks] : rb.hwp[ks]), &s4, &c4);
+                st_base[12 * ks + 9] = c4;
+                st_base[12 * ks + 10] = s4;
             }
-            SampleState x;
-            quat_to_matrix(q0, q1, q2, q3, x.v);
-            x.v[9] = c4;
-            x.v[10] = s4;
-            x.v[11] = 0.0;
-            if constexpr (TMA)
-                *reinterpret_cast<SampleState*>(tw.st[lane]) = x;
-            else
-                sm.st[lane] = x;
         }
         const unsigned pmask = __ballot_sync(0xffffffffu, pixelise_me);
-        // det flags of the lane's rows -> one bit per sample (bit k: sample k is det-flagged)
-        unsigned fmask[DPL];
+        const unsigned keep = ((1u << cur.nb) - 1u) << cur.k0;  // samples of the block processed (nb <= 16)
+        // The staged TOD of det-flagged samples (and, with debug outputs, of shared-flagged
+        // samples, which run through det_sample without a pixel) is zeroed in shared memory, so
+        // the per-sample loop needs no flag test: those samples add exactly 0 to the map.
 #pragma unroll
         for (int j = 0; j < DPL; ++j) {
-            fmask[j] = 0u;
             const int row = lane + 32 * j;
+            unsigned zm = DEBUG ? (~pmask & keep) : 0u;
             if (have_dflags && row < cur.nrows) {
                 const unsigned rep = dmask * 0x01010101u;
-                const unsigned keep = ((1u << cur.nb) - 1u) << cur.k0;  // nb <= 16
+                unsigned bits = 0u;  // bit k: sample k of the box is det-flagged
                 if constexpr (TMA) {
                     const uint4 f = *reinterpret_cast<const uint4*>(tw.flg[p][row]);
                     const unsigned fw[4] = {f.x, f.y, f.z, f.w};
-                    unsigned bits = 0u;
 #pragma unroll
                     for (int w = 0; w < 4; ++w) {
                         const unsigned v = __vcmpne4(fw[w] & rep, 0u);
                         bits |= ((v & 0x01010101u) * 0x01020408u >> 24 & 0xfu) << (4 * w);
                     }
-                    fmask[j] = bits & keep;
                 } else {
                     const int foff =
                         (int)(reinterpret_cast<uintptr_t>(a.det_flags + (cur.d0 + row) * a.n_samp + cur.s0) & 3);
-                    unsigned bits = 0u;  // bit b: byte b of the 20-byte window is flagged
 #pragma unroll
-                    for (int w = 0; w < 5; ++w) {
+                    for (int w = 0; w < 5; ++w) {  // bit b: byte b of the 20-byte window is flagged
                         const unsigned v = __vcmpne4(*reinterpret_cast<const unsigned*>(&rb.flg[row][4 * w]) & rep, 0u);
                         bits |= ((v & 0x01010101u) * 0x01020408u >> 24 & 0xfu) << (4 * w);
                     }
-                    fmask[j] = (bits >> foff) & keep;
+                    bits >>= foff;
                 }
+                zm |= bits & keep;
+            }
+            while (zm) {
+                const int k = __ffs(zm) - 1;
+                zm &= zm - 1;
+                if constexpr (TMA)
+                    *reinterpret_cast<double*>(reinterpret_cast<unsigned char*>(&tw.tod[p][0][0]) +
+                                               (row_swz ^ ((unsigned)k << 3))) = 0.0;
+                else
+                    rb.tod[row][k] = 0.0;
             }
         }
         __syncwarp();
 
-        const double* st_base = TMA ? &tw.st[0][0] : &sm.st[0].v[0];
-        const unsigned char* tod_tile = reinterpret_cast<const unsigned char*>(&tw.tod[p][0][0]);
+        // TMA tile: the tile is 1 KB-aligned and row r starts at r * 128, so the swizzled address
+        // of (lane, k) is (tile + row_swz) ^ (8 k): one LOP3 per sample.
+        const unsigned tod_row = smem_u32(&tw.tod[p][0][0]) + row_swz;
         unsigned bit = 1u << cur.k0;  // 1 << k
 #pragma unroll kKUnroll
         for (int k = cur.k0; k < cur.k0 + cur.nb; ++k, bit <<= 1) {
@@ -634,30 +684,27 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
                 x[i + 1] = t2.y;
             }
             double tod[DPL];
-            bool dflag[DPL];
 #pragma unroll
             for (int j = 0; j < DPL; ++j) {
-                const int row = lane + 32 * j;
                 if constexpr (TMA)
-                    tod[j] = *reinterpret_cast<const double*>(tod_tile + (row_swz ^ ((unsigned)k << 3)));
+                    asm volatile("ld.shared.f64 %0, [%1];" : "=d"(tod[j]) : "r"(tod_row ^ ((unsigned)k << 3)));
                 else
-                    tod[j] = rb.tod[row][k];
-                dflag[j] = fmask[j] & bit;
+                    tod[j] = rb.tod[lane + 32 * j][k];
             }
             // fold the previous sample while those shared-memory loads are in flight
 #pragma unroll
-            for (int j = 0; j < DPL; ++j) aggregate<NNZ, P>(sl[j], a);
+            for (int j = 0; j < DPL; ++j) aggregate<NEST, NNZ, WIDE>(sl[j], a, g);
 #pragma unroll
             for (int j = 0; j < DPL; ++j)
-                det_sample<NEST, NNZ, HWP, DEBUG, WIDE>(sl[j], x, pixelise, tod[j], dflag[j], g, a,
-                                                        cur.d0 + lane + 32 * j, cur.s0 + k);
+                det_sample<NEST, NNZ, HWP, DEBUG, WIDE>(sl[j], x, pixelise, tod[j], g, a, cur.d0 + lane + 32 * j,
+                                                        cur.s0 + k);
         }
 
         if (nxt.item != cur.item) {
 #pragma unroll
             for (int j = 0; j < DPL; ++j) {
-                aggregate<NNZ, P>(sl[j], a);
-                if (sl[j].run_pix >= 0) flush<NNZ, P>(sl[j].run_pix, sl[j].run_loc, sl[j].r0, sl[j].r1, sl[j].r2, a);
+                aggregate<NEST, NNZ, WIDE>(sl[j], a, g);
+                flush<NNZ, WIDE>(sl[j].run_loc, sl[j].run_lp, sl[j].r0, sl[j].r1, sl[j].r2, a);
             }
             if (nxt.item < 0) break;
 #pragma unroll
@@ -787,9 +834,13 @@ cudaError_t launch_k(const WorkList& wl, const FusedArgs& a, const TmaMaps& tm, 
 template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL>
 cudaError_t launch_t(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
     TmaMaps tm;
-    if (DPL == 1 && make_tma_maps(a, &tm)) {
-        t_fused_path = "tma";
-        return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, 1, true>(wl, a, tm, sched, st);
+    if constexpr (kBlk == 16) {
+        if (DPL == 1 && make_tma_maps(a, &tm)) {
+            t_fused_path = "tma";
+            return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, 1, true>(wl, a, tm, sched, st);
+        }
+    } else {
+        t_fused_path = "cp.async (8-sample blocks)";
     }
     std::memset(&tm, 0, sizeof(tm));
     return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, DPL, false>(wl, a, tm, sched, st);
