@@ -56,6 +56,9 @@ constexpr int kRowStep = 32 / kBlk;  // TOD rows staged per cp.async instruction
 #define TB_KUNROLL 1
 #endif
 constexpr int kKUnroll = TB_KUNROLL;  // unroll of the per-sample loop
+#ifndef TB_PAIR
+#define TB_PAIR 0
+#endif
 constexpr int kPad = kBlk + 1;
 
 // per-sample state: B[0..8], c4, s4, mode (as a double: 1 pixelise, 2 shared-flagged)
@@ -314,72 +317,98 @@ __device__ __forceinline__ void load_slot(Slot<P>& sl, const FusedArgs& a, int64
     sl.ok = ok;
 }
 
+// The straight-line fp64 part of one det-sample (A1 -> direction, A3 weights and the A2
+// longitude): no branches, so two of them can be interleaved by the scheduler (pair loop).
+struct StageA {
+    double dx, dy, dz, tt;
+    double cw, sw, invr;  // r cos 2(psi + 2 chi), r sin 2(psi + 2 chi), 1/r
+};
+
+template <int NNZ, bool HWP, typename P>
+__device__ __forceinline__ StageA stage_a(const Slot<P>& sl, const double* x) {
+    StageA o;
+    o.dx = x[0] * sl.u0 + x[1] * sl.u1 + x[2] * sl.u2;
+    o.dy = x[3] * sl.u0 + x[4] * sl.u1 + x[5] * sl.u2;
+    o.dz = x[6] * sl.u0 + x[7] * sl.u1 + x[8] * sl.u2;
+    o.cw = o.sw = o.invr = 0.0;
+    if (NNZ == 3) {
+        const double bx = x[6] * sl.v0 + x[7] * sl.v1 + x[8] * sl.v2;
+        const double by = -(x[6] * sl.w0 + x[7] * sl.w1 + x[8] * sl.w2);
+#ifdef TB_X_NOATAN
+        o.tt = fabs(o.dx) * 3.9; o.cw = bx; o.sw = by; o.invr = 1.0;  // ablation: no longitude/weights arithmetic
+#else
+        o.tt = lon_pol_raw(o.dx, o.dy, bx, by, o.cw, o.sw, o.invr);  // one shared reciprocal
+#endif
+        if (HWP) {
+            const double c4 = x[9], s4 = x[10];
+            const double cq = o.cw * c4 - o.sw * s4;
+            const double sq = o.sw * c4 + o.cw * s4;
+            o.cw = cq;
+            o.sw = sq;
+        }
+    } else {
+        o.tt = quarter_turns(o.dx, o.dy);
+    }
+    return o;
+}
+
+// The HEALPix floors and integer part (branches: equatorial belt / caps): the run key.
+template <bool NEST, bool WIDE>
+__device__ __forceinline__ typename PixT<WIDE>::T stage_b(const StageA& o, bool pixelise, bool ok,
+                                                         const HealpixGeom& g) {
+    using P = typename PixT<WIDE>::T;
+    P key = -1;
+    if (pixelise) {
+        if constexpr (WIDE)
+            key = (P)loc2pix<NEST, int64_t>(g, o.dz, o.tt, o.dx, o.dy);
+        else
+#ifdef TB_X_NOPIX
+            key = (P)((int)(o.tt * 1000.0) & 0xffff);  // ablation: no HEALPix integer/floor logic
+#else
+            key = (P)loc2key32<NEST>(g, o.dz, o.tt, o.dx, o.dy);
+#endif
+    }
+    if (!ok) key = -1;
+    return key;
+}
+
+// The A4 contribution of a det-sample, pending until aggregate() folds it into the run.
+// Det-flagged samples keep their key (they mark hit submaps, as A2 does) but add 0 (their
+// staged tod is 0); so does every sample without a key (aggregate() adds unconditionally).
+template <int NNZ, typename P>
+__device__ __forceinline__ void set_pending(Slot<P>& sl, const StageA& o, P key, double tod) {
+    sl.pend_key = key;
+    sl.p0 = tod * sl.s_cal;
+    if (NNZ == 3) {
+        const double t = (tod * sl.s_eta) * o.invr;
+        sl.p1 = t * o.cw;
+        sl.p2 = t * o.sw;
+    }
+}
+
 // One det-sample of slot `sl` with the per-sample state x.  `tod` is already 0 for det-flagged
 // samples (and, with debug outputs, shared-flagged ones): the block prologue zeroes them in the
-// staged tile, so no per-sample flag test is needed here.
+// staged tile, so no per-sample flag test is needed here.  Its contribution is folded into the
+// lane's run by aggregate() one sample LATER, so that work overlaps the next sample's loads.
 template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE>
 __device__ __forceinline__ void det_sample(Slot<typename PixT<WIDE>::T>& sl, const double* x, bool pixelise,
                                            double tod, const HealpixGeom& g, const FusedArgs& a, int64_t d,
                                            int64_t s) {
     using P = typename PixT<WIDE>::T;
-    const double dx = x[0] * sl.u0 + x[1] * sl.u1 + x[2] * sl.u2;
-    const double dy = x[3] * sl.u0 + x[4] * sl.u1 + x[5] * sl.u2;
-    const double dz = x[6] * sl.u0 + x[7] * sl.u1 + x[8] * sl.u2;
-    // The weight chain and the longitude chain are independent and branch-free: they are
-    // written into one basic block so the scheduler can interleave them (latency-bound code).
-    double cw = 0.0, sw = 0.0, invr = 0.0, tt;  // r cos 2(psi + 2 chi), r sin 2(psi + 2 chi), 1/r
-    if (NNZ == 3) {
-        const double bx = x[6] * sl.v0 + x[7] * sl.v1 + x[8] * sl.v2;
-        const double by = -(x[6] * sl.w0 + x[7] * sl.w1 + x[8] * sl.w2);
-#ifdef TB_X_NOATAN
-        tt = fabs(dx) * 3.9; cw = bx; sw = by; invr = 1.0;  // ablation: no longitude/weights arithmetic
-#else
-        tt = lon_pol_raw(dx, dy, bx, by, cw, sw, invr);  // one shared reciprocal
-#endif
-        if (HWP) {
-            const double c4 = x[9], s4 = x[10];
-            const double cq = cw * c4 - sw * s4;
-            const double sq = sw * c4 + cw * s4;
-            cw = cq;
-            sw = sq;
-        }
-    } else {
-        tt = quarter_turns(dx, dy);
-    }
-    P key = -1;
-    if (pixelise) {
-        if constexpr (WIDE)
-            key = (P)loc2pix<NEST, int64_t>(g, dz, tt, dx, dy);
-        else
-#ifdef TB_X_NOPIX
-            key = (P)((int)(tt * 1000.0) & 0xffff);  // ablation: no HEALPix integer/floor logic
-#else
-            key = (P)loc2key32<NEST>(g, dz, tt, dx, dy);
-#endif
-    }
-    if (!sl.ok) key = -1;
+    const StageA o = stage_a<NNZ, HWP, P>(sl, x);
+    const P key = stage_b<NEST, WIDE>(o, pixelise, sl.ok, g);
     if (DEBUG && sl.ok) {
-        const int64_t o = d * a.n_samp + s;
-        if (a.pixels_out) a.pixels_out[o] = key < 0 ? (int64_t)-1 : (int64_t)key_to_pix<NEST, WIDE>(key, g);
+        const int64_t off = d * a.n_samp + s;
+        if (a.pixels_out) a.pixels_out[off] = key < 0 ? (int64_t)-1 : (int64_t)key_to_pix<NEST, WIDE>(key, g);
         if (a.weights_out) {
-            a.weights_out[o * NNZ] = a.cal;
+            a.weights_out[off * NNZ] = a.cal;
             if (NNZ == 3) {
-                a.weights_out[o * NNZ + 1] = sl.etacal * (cw * invr);
-                a.weights_out[o * NNZ + 2] = sl.etacal * (sw * invr);
+                a.weights_out[off * NNZ + 1] = sl.etacal * (o.cw * o.invr);
+                a.weights_out[off * NNZ + 2] = sl.etacal * (o.sw * o.invr);
             }
         }
     }
-    // A4 contribution of this det-sample; it is folded into the lane's run by aggregate()
-    // one sample LATER, so that work overlaps the shared-memory loads of the next sample.
-    // Det-flagged samples keep their key (they mark hit submaps, as A2 does) but add 0 (their
-    // staged tod is 0); so does every sample without a key (aggregate() adds unconditionally).
-    sl.pend_key = key;
-    sl.p0 = tod * sl.s_cal;
-    if (NNZ == 3) {
-        const double t = (tod * sl.s_eta) * invr;
-        sl.p1 = t * cw;
-        sl.p2 = t * sw;
-    }
+    set_pending<NNZ, P>(sl, o, key, tod);
 }
 
 // Fold the pending contribution into the run (run-length aggregation along time).  Lanes
@@ -458,6 +487,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
                                                                          unsigned long long* __restrict__ sched,
                                                                          const __grid_constant__ TmaMaps tm) {
     static_assert(!TMA || (DPL == 1 && kBlk == 16), "the TMA path stages 32 x 16 tiles");
+    constexpr bool PAIR = TB_PAIR && TMA && !DEBUG;
     using P = typename PixT<WIDE>::T;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int lane = threadIdx.x & 31;
@@ -632,7 +662,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
 #pragma unroll
         for (int j = 0; j < DPL; ++j) {
             const int row = lane + 32 * j;
-            unsigned zm = DEBUG ? (~pmask & keep) : 0u;
+            unsigned zm = (DEBUG || PAIR) ? (~pmask & keep) : 0u;
             if (have_dflags && row < cur.nrows) {
                 const unsigned rep = dmask * 0x01010101u;
                 unsigned bits = 0u;  // bit k: sample k of the box is det-flagged
@@ -671,9 +701,39 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
         // TMA tile: the tile is 1 KB-aligned and row r starts at r * 128, so the swizzled address
         // of (lane, k) is (tile + row_swz) ^ (8 k): one LOP3 per sample.
         const unsigned tod_row = smem_u32(&tw.tod[p][0][0]) + row_swz;
-        unsigned bit = 1u << cur.k0;  // 1 << k
+        int k = cur.k0;
+        const int k_end = cur.k0 + cur.nb;
+#if TB_PAIR
+        if constexpr (PAIR) {
+            // two samples per iteration: their branch-free fp64 parts (stage_a) are issued
+            // back to back so the scheduler interleaves two independent dependency chains;
+            // shared-flagged samples run through with no key and a zeroed tod
+            for (; k + 1 < k_end; k += 2) {
+                double x0[12], x1[12];
+#pragma unroll
+                for (int i = 0; i < ((HWP && NNZ == 3) ? 12 : 10); i += 2) {
+                    const double2 t0 = *reinterpret_cast<const double2*>(st_base + 12 * k + i);
+                    const double2 t1 = *reinterpret_cast<const double2*>(st_base + 12 * k + 12 + i);
+                    x0[i] = t0.x; x0[i + 1] = t0.y;
+                    x1[i] = t1.x; x1[i + 1] = t1.y;
+                }
+                double tod0, tod1;
+                asm volatile("ld.shared.f64 %0, [%1];" : "=d"(tod0) : "r"(tod_row ^ ((unsigned)k << 3)));
+                asm volatile("ld.shared.f64 %0, [%1];" : "=d"(tod1) : "r"(tod_row ^ ((unsigned)(k + 1) << 3)));
+                const StageA o0 = stage_a<NNZ, HWP, P>(sl[0], x0);
+                const StageA o1 = stage_a<NNZ, HWP, P>(sl[0], x1);
+                aggregate<NEST, NNZ, WIDE>(sl[0], a, g);
+                const P key0 = stage_b<NEST, WIDE>(o0, (pmask >> k) & 1u, sl[0].ok, g);
+                set_pending<NNZ, P>(sl[0], o0, key0, tod0);
+                aggregate<NEST, NNZ, WIDE>(sl[0], a, g);
+                const P key1 = stage_b<NEST, WIDE>(o1, (pmask >> (k + 1)) & 1u, sl[0].ok, g);
+                set_pending<NNZ, P>(sl[0], o1, key1, tod1);
+            }
+        }
+#endif
+        unsigned bit = 1u << k;  // 1 << k
 #pragma unroll kKUnroll
-        for (int k = cur.k0; k < cur.k0 + cur.nb; ++k, bit <<= 1) {
+        for (; k < k_end; ++k, bit <<= 1) {
             const bool pixelise = pmask & bit;
             if (!DEBUG && !pixelise) continue;  // shared-flagged sample: nothing to add (uniform)
             double x[12];
