@@ -316,8 +316,18 @@ def main():
     except (OSError, ValueError):
         pass
     hbm_peak = float(peaks.get("hbm_gbs", 6650.0))
+    # DRAM traffic of one launch of the fused kernel, from the committed ncu --set full capture
+    # of this workload (profiles/traffic.json; ncu never runs inside the bench), else null
+    traffic, traffic_src = None, None
+    try:
+        tr = json.load(open(os.path.join(ROOT, "profiles", "traffic.json"))).get(args.workload)
+        if tr:
+            traffic, traffic_src = float(tr["dram_bytes_per_launch"]), tr["source"]
+    except (OSError, ValueError, KeyError):
+        pass
     roofline = {"bound": "alu", "achieved": ach_tflops, "peak": peak_tflops, "unit": "TFLOP/s",
-                "frac": ach_tflops / peak_tflops, "traffic": None,
+                "frac": ach_tflops / peak_tflops, "traffic": traffic, "traffic_unit": "B/launch",
+                "traffic_source": traffic_src,
                 "kernel": "pointing_to_map_kernel (fused A1-A4)", "kernel_ms": kern_ms,
                 "f_alg_per_det_sample": F_ALG,
                 "peak_note": f"fp64 pipe: {SMS} SM x {DFMA_PER_SM_PER_CLK} DFMA/clk x 2 x {clk:.0f} MHz (derived, "
