@@ -526,3 +526,42 @@ def test_template_offsets_gpu(step):
     out = torch.zeros(n_det * n_amp, dtype=torch.float64, device=DEV)
     binding.template_offset_apply_diag_precond(_cuda(var, torch.float64), ag, out)
     np.testing.assert_array_equal(out.cpu().numpy(), oracle.template_offset_apply_diag_precond(var, ag.cpu().numpy()))
+
+
+@pytest.mark.parametrize("nside,nest", [(1 << 13, True), (1 << 13, False), (1 << 20, True)])
+def test_fused_incremental_longitude_wraps_and_poles(nside, nest):
+    """The fused kernel carries the longitude incrementally along each detector's samples
+    (DESIGN.md "Fused kernel"): boresights that circle the pole (the quarter-turn longitude
+    wraps 4 -> 0 every ~600 samples, steps of 0.01 rad: the series path), that cross it (the
+    step exceeds the series range: the full-arctangent fallback) and a slow drift (long series
+    chains) give the oracle's pixels up to near-boundary samples, at fine pixelisations."""
+    n_samp = 6000
+    w = synth.make_workload("c1", n_samp=n_samp, nside=nside, nest=nest, nnz=3)
+    t = np.arange(n_samp, dtype=np.float64)
+    third = n_samp // 3
+    a, b, c = t[:third], t[third:2 * third], t[2 * third:]
+    mats = np.concatenate([
+        # circle at colatitude 0.05 rad: phi advances 0.01 rad per sample
+        synth.matmul_chain(synth.rot_axis("z", 0.01 * a), synth.rot_axis("y", np.full_like(a, 0.05))),
+        # great circle through both poles, 2e-3 rad per sample
+        synth.rot_axis("x", 2e-3 * (b - third) - 0.3),
+        # slow drift near the equator
+        synth.matmul_chain(synth.rot_axis("z", 1e-5 * c + 1.0), synth.rot_axis("y", np.full_like(c, 1.2))),
+    ])
+    w.boresight = synth.matrix_to_quat(mats)
+    w.intervals = [(0, n_samp - 1)]
+    w.n_pix_submap = (nside // 16) ** 2
+    quats = oracle.pointing_detector(w.fp_quats, w.boresight, w.intervals)
+    po, hits = oracle.pixels_healpix(quats, w.intervals, nside, nest, w.n_pix_submap)
+    dw = DeviceWorkload.upload(w, DEV, alloc_map=False)
+    dw.global2local = torch.full((w.n_submap,), -1, dtype=torch.int64, device=DEV)
+    dw.zmap = torch.zeros((1, 1, 3), dtype=torch.float64, device=DEV)
+    pix_g = torch.full((w.n_det, w.n_samp), -7, dtype=torch.int64, device=DEV)
+    wts_g = torch.zeros((w.n_det, w.n_samp, 3), dtype=torch.float64, device=DEV)
+    dw.pointing_to_map(pixels_out=pix_g, weights_out=wts_g)
+    torch.cuda.synchronize()
+    classify_pixel_mismatches(pix_g.cpu().numpy(), po, _probe(w), nside, nest, w.n_det * n_samp)
+    np.testing.assert_array_equal(dw.hit_submaps.cpu().numpy(), hits)
+    wo = oracle.stokes_weights_iqu(quats, w.intervals, w.epsilon, w.cal, hwp=w.hwp)
+    eta_cal = (1 - w.epsilon) / (1 + w.epsilon) * w.cal
+    check_weights(wts_g.cpu().numpy(), wo, _sin_theta(quats), eta_cal, w.cal, np.ones((w.n_det, n_samp), bool))
