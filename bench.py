@@ -57,8 +57,10 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--soak", type=float, default=1.0, help="seconds of untimed steps before timing (clocks)")
-    ap.add_argument("--reduce", default="auto", choices=["auto", "dense", "packed"],
-                    help="N>1 map reduction: dense all_reduce, or all_reduce of the union of hit submaps")
+    ap.add_argument("--reduce", default="auto", choices=["auto", "dense", "packed", "scatter"],
+                    help="N>1 map reduction: dense all_reduce, all_reduce of the union of hit submaps "
+                         "(packed), or the sparse distributed map domain: a map stored for the union of hit "
+                         "submaps only, reduce_scatter to per-rank owned blocks (scatter, SURVEY 8(f) f3)")
     return ap.parse_args()
 
 
@@ -240,7 +242,20 @@ def main():
     call = lib.toast_pointing_to_map
 
     packed = args.reduce == "packed" or (args.reduce == "auto" and dw.zmap.numel() * 8 > (256 << 20))
+    scatter = args.reduce == "scatter"
     reduced = [0]
+    own = None
+    if scatter:
+        # pixel distribution (untimed setup, as TOAST computes it once per data set): the union
+        # over ranks of the hit submaps, from one pass of the fused entry; then the compact map
+        dw.pointing_to_map()
+        tdist.union_hit_submaps(dw.hit_submaps)
+        g2l_c, n_hit = tdist.compact_global2local(dw.hit_submaps)
+        own = tdist.MapOwnership.make(n_hit, world)
+        dw.global2local = g2l_c
+        dw.zmap = tdist.alloc_compact_map(own, w.n_pix_submap, w.nnz, "cuda")
+        raw = dw.raw_args(stream)
+        torch.cuda.synchronize()
 
     def step(k0=None, k1=None):
         dw.zmap.zero_()
@@ -254,7 +269,9 @@ def main():
         if k1 is not None:
             k1.record(stream)
         if world > 1:
-            if packed:
+            if scatter:
+                _, reduced[0] = tdist.reduce_scatter_map(dw.zmap, own)
+            elif packed:
                 tdist.union_hit_submaps(dw.hit_submaps)
                 _, reduced[0] = tdist.reduce_map(dw.zmap, hit_submaps=dw.hit_submaps, global2local=dw.global2local)
             else:
@@ -352,8 +369,11 @@ def main():
                            "parallelism": f"dp{world} (one observation per rank + NCCL all-reduce of the map)"
                            if world > 1 else "single GPU",
                            "step": "zero map + toast_pointing_to_map" + (
-                               (" + all_reduce(hit submaps, MAX) + packed all_reduce(map)" if packed
+                               (" + reduce_scatter(compact map of the hit submaps)" if scatter
+                                else " + all_reduce(hit submaps, MAX) + packed all_reduce(map)" if packed
                                 else " + all_reduce(map)") if world > 1 else ""),
+                           "map_domain": (f"compact: {own.n_hit} hit submaps of {w.n_submap}" if scatter
+                                          else f"dense: {w.n_submap} submaps"),
                            "allreduce_bytes_per_step": reduced[0],
                            "staging": binding.last_fused_path()},
                 "clocks": clocks, "gpu_launches": args.steps, "roofline": roofline}

@@ -419,7 +419,11 @@ __device__ __forceinline__ int loc2pix32(const HealpixGeom& g, double dz, double
 // packing that costs two IMADs per det-sample instead of the bit interleave, which
 // key_to_pix32 applies once per run.  Same floors, in the same order and rounding, as
 // loc2pix32.
-template <bool NEST>
+// OFF: tt is the longitude in quarter turns PLUS ONE, unwrapped, anywhere in (0.18, 5.82) (the
+// fused kernel's incremental longitude, see stage_a): every floor argument stays positive, the
+// equatorial jp, jm and the cap ip carry an extra N (resp. ir), and the face / ring position is
+// folded back modulo 4 quarter turns here — no per-sample wrap of tt.
+template <bool NEST, bool OFF = false>
 __device__ __forceinline__ int loc2key32(const HealpixGeom& g, double dz, double tt, double dx, double dy) {
     const double za = fabs(dz);
     const int nside = (int)g.nside;
@@ -433,13 +437,18 @@ __device__ __forceinline__ int loc2key32(const HealpixGeom& g, double dz, double
             const int nl4 = 4 * nside;
             const int ir = nside + 1 + jp - jm;
             const int kshift = 1 - (ir & 1);
-            const int t1 = jp + jm - nside + kshift + 1 + 2 * nl4;
+            const int t1 = jp + jm - (OFF ? 3 : 1) * nside + kshift + 1 + 2 * nl4;
             const int ip = (t1 >> 1) & (nl4 - 1);
             return (int)g.ncap + nl4 * (ir - 1) + ip;
         } else {
-            const int ifp = jp >> g.order;
-            const int ifm = jm >> g.order;
-            const int face = (ifp == ifm) ? (ifp | 4) : ((ifp < ifm) ? ifp : (ifm + 8));
+            int ifp = jp >> g.order;
+            int ifm = jm >> g.order;
+            int face;
+            if (OFF) {  // ifp, ifm in 0..6 stand for faces (ifp - 1) mod 4, (ifm - 1) mod 4
+                face = (ifp == ifm) ? (((ifp + 3) & 3) | 4) : ((ifp < ifm) ? ((ifp + 3) & 3) : (((ifm + 3) & 3) | 8));
+            } else {
+                face = (ifp == ifm) ? (ifp | 4) : ((ifp < ifm) ? ifp : (ifm + 8));
+            }
             const int ix = jm & m;
             const int iy = (jp & m) ^ m;  // nside - 1 - (jp & (nside - 1))
             return (face * nside + iy) * nside + ix;
@@ -458,12 +467,17 @@ __device__ __forceinline__ int loc2key32(const HealpixGeom& g, double dz, double
         const int jm = floor_nonneg(__dmul_rn(__dsub_rn(1.0, tp), tmp));
         const int ir = jp + jm + 1;
         int ip = floor_nonneg(__dmul_rn(tt, small_int_to_double(ir)));
+        if (OFF) {
+            ip -= ir;  // in [-0.82 ir, 4.82 ir)
+            if (ip < 0) ip += 4 * ir;
+        }
         if (ip >= 4 * ir) ip -= 4 * ir;
         return (dz > 0.0) ? 2 * ir * (ir - 1) + ip : (int)g.npix - 2 * ir * (ir + 1) + ip;
     } else {
         int ntt = floor_nonneg(tt);
-        if (ntt > 3) ntt = 3;
+        if (!OFF && ntt > 3) ntt = 3;
         const double tp = __dsub_rn(tt, small_int_to_double(ntt));
+        if (OFF) ntt = (ntt + 3) & 3;
         int jp = floor_nonneg(__dmul_rn(tp, tmp));
         int jm = floor_nonneg(__dmul_rn(__dsub_rn(1.0, tp), tmp));
         if (jp > m) jp = m;

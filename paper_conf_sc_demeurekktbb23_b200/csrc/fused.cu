@@ -59,14 +59,17 @@ constexpr int kRowStep = 32 / kBlk;  // TOD rows staged per cp.async instruction
 #define TB_KUNROLL 1
 #endif
 constexpr int kKUnroll = TB_KUNROLL;  // unroll of the per-sample loop
-#ifndef TB_PAIR
-#define TB_PAIR 0
-#endif
 #ifndef TB_INCR
 #define TB_INCR 1  // incremental longitude along each detector's samples (see stage_a)
 #endif
-#ifndef TB_PARK
-#define TB_PARK 0  // block-end flush of finished runs (see aggregate; measured: +15% C3, -20% C4)
+#ifndef TB_FOLD
+#define TB_FOLD 1  // det_scale (and eta cal) applied once per run at the flush, not per det-sample
+#endif
+#ifndef TB_TTOFF
+#define TB_TTOFF 1  // 32-bit keys: longitude carried as tt + 1 without wrapping (see stage_a)
+#endif
+#ifndef TB_SMCACHE
+#define TB_SMCACHE 0  // run start: per-lane submap cache (measured on B200: -1.5% C2, -0.5% C3; off)
 #endif
 constexpr int kPad = kBlk + 1;
 
@@ -231,97 +234,6 @@ __device__ __forceinline__ typename PixT<WIDE>::T key_to_pix(typename PixT<WIDE>
     }
 }
 
-// A run starts: mark its submap hit (as A2 does) and issue the global2local lookup now, so
-// the load latency is hidden behind the run's samples instead of stalling the flush.  The hit
-// flag is stored only when the lane's submap CHANGES: thousands of warps re-writing the same
-// few bytes of hit_submaps serialise in L2 and cost as much as the whole computation.  `lp`
-// receives the pixel's index inside its submap.
-template <bool NEST, bool WIDE>
-__device__ __forceinline__ int64_t start_run(typename PixT<WIDE>::T key, const FusedArgs& a, const HealpixGeom& g,
-                                             typename PixT<WIDE>::T& last_sm, typename PixT<WIDE>::T& lp) {
-    using P = typename PixT<WIDE>::T;
-    const MapGeom& mg = a.map;
-    const P pix = key_to_pix<NEST, WIDE>(key, g);
-    P sm;
-    if (mg.sm_shift >= 0) {
-        sm = pix >> mg.sm_shift;
-        lp = pix & (P)(mg.n_pix_submap - 1);
-    } else {
-        sm = pix / (P)mg.n_pix_submap;
-        lp = pix - sm * (P)mg.n_pix_submap;
-    }
-#ifndef TB_X_NOHIT
-    if (a.hit_submaps && sm != last_sm) {
-        a.hit_submaps[sm] = 1;
-        last_sm = sm;
-    }
-#endif
-#ifdef TB_X_NOG2L
-    return sm;
-#else
-    return __ldg(&mg.global2local[sm]);
-#endif
-}
-
-// A run ends: one fp64 red per Stokes component (nothing if the submap has no storage).  Up to
-// nside 8192 the map element index fits 32 bits (< 12 * 8192^2 pixels), so the address is one
-// IMAD + one IMAD.WIDE.U32.
-template <int NNZ, bool WIDE>
-__device__ __forceinline__ void flush(int64_t loc, typename PixT<WIDE>::T lp, double a0, double a1, double a2,
-                                      const FusedArgs& a) {
-    if (loc < 0) return;
-    double* dst;
-    if constexpr (WIDE) {
-        dst = a.zmap + (loc * a.map.n_pix_submap + lp) * NNZ;
-    } else {
-        const unsigned idx = (unsigned)loc * (unsigned)a.map.n_pix_submap + (unsigned)lp;
-        dst = a.zmap + (size_t)idx * NNZ;
-    }
-    atomicAdd(dst, a0);
-    if (NNZ == 3) {
-        atomicAdd(dst + 1, a1);
-        atomicAdd(dst + 2, a2);
-    }
-}
-
-// A finished run, flushed in one go: its pixel, the submap hit mark, the global2local lookup and
-// one fp64 red per Stokes component (PARK mode: at block ends, when the load latency is hidden by
-// the other warps).
-// With MapGeom::sm_fast the lane caches the submap of its last flush (smk: its key bits, loc:
-// its global2local entry): a run in the same submap needs neither the pixel, the hit mark nor
-// the global2local load — only the pixel's index inside the submap — so a flush costs ~15
-// instructions and exposes no load latency.
-template <bool NEST, int NNZ, bool WIDE>
-__device__ __forceinline__ void flush_run(typename PixT<WIDE>::T key, double a0, double a1, double a2,
-                                          const FusedArgs& a, const HealpixGeom& g,
-                                          typename PixT<WIDE>::T& last_sm, int& c_smk, int64_t& c_loc) {
-    if constexpr (!WIDE) {
-        const MapGeom& mg = a.map;
-        if (mg.sm_fast) {
-            const int smk = NEST ? (key & mg.smk_mask) : (key >> mg.sm_shift);
-            if (smk != c_smk) {
-                const int pix = key_to_pix<NEST, WIDE>(key, g);
-                const int sm = pix >> mg.sm_shift;
-                if (a.hit_submaps) a.hit_submaps[sm] = 1;
-                c_loc = __ldg(&mg.global2local[sm]);
-                c_smk = smk;
-            }
-            int lp;
-            if (NEST) {
-                const int bm = (1 << mg.lp_bits) - 1;
-                lp = (int)interleave16((uint32_t)(key & bm), (uint32_t)((key >> g.order) & bm));
-            } else {
-                lp = key & ((1 << mg.sm_shift) - 1);
-            }
-            flush<NNZ, WIDE>(c_loc, lp, a0, a1, a2, a);
-            return;
-        }
-    }
-    typename PixT<WIDE>::T lp;
-    const int64_t loc = start_run<NEST, WIDE>(key, a, g, last_sm, lp);
-    flush<NNZ, WIDE>(loc, lp, a0, a1, a2, a);
-}
-
 template <typename P>
 struct Slot {
     double u0, u1, u2, v0, v1, v2, w0, w1, w2;
@@ -331,17 +243,102 @@ struct Slot {
     P run_key;            // key of the run being aggregated (-1: none)
     P run_lp;             // its pixel's index inside the submap
     int64_t run_loc;      // global2local of the run's submap, LOADED WHEN THE RUN STARTS
-    P last_sm;            // last submap this lane marked in hit_submaps
+    P last_sm;            // last submap this lane marked in hit_submaps (generic path)
+    int c_smk;            // MapGeom::sm_fast: submap key bits of the last run start
+    int64_t c_loc;        //   and its global2local entry
     double r0, r1, r2;
     P pend_key;           // pending (not yet aggregated) det-sample
     double p0, p1, p2;
-    P park_key;           // PARK mode: a finished run waiting for the block-end flush (-1: none)
-    double q0, q1, q2;
     double px, py, ptt;   // INCR mode: projected direction and tt of the lane's previous sample
-    int c_smk;            // PARK mode with MapGeom::sm_fast: submap key bits of the last flush
-    int64_t c_loc;        //   and its global2local entry
     bool ok;
 };
+
+// A run starts: mark its submap hit (as A2 does) and issue the global2local lookup now, so
+// the load latency is hidden behind the run's samples instead of stalling the flush.  The hit
+// flag is stored only when the lane's submap CHANGES: thousands of warps re-writing the same
+// few bytes of hit_submaps serialise in L2 and cost as much as the whole computation.
+// With MapGeom::sm_fast (32-bit keys, power-of-two submaps) the submap is read off the key bits
+// and compared with the lane's last one: a run in the same submap (nearly all of them) needs
+// neither the pixel, the hit mark nor the global2local load — only the pixel's index inside the
+// submap.  Sets sl.run_loc (-1: the submap has no storage) and sl.run_lp.
+template <bool NEST, bool WIDE>
+__device__ __forceinline__ void start_run(typename PixT<WIDE>::T key, const FusedArgs& a, const HealpixGeom& g,
+                                          Slot<typename PixT<WIDE>::T>& sl) {
+    using P = typename PixT<WIDE>::T;
+    const MapGeom& mg = a.map;
+#if TB_SMCACHE
+    if constexpr (!WIDE) {
+        if (mg.sm_fast) {
+            const int smk = NEST ? (key & mg.smk_mask) : (key >> mg.sm_shift);
+            if (smk != sl.c_smk) {
+                const int sm = key_to_pix<NEST, WIDE>(key, g) >> mg.sm_shift;
+#ifndef TB_X_NOHIT
+                if (a.hit_submaps) a.hit_submaps[sm] = 1;
+#endif
+                sl.c_loc = __ldg(&mg.global2local[sm]);
+                sl.c_smk = smk;
+            }
+            if (NEST) {
+                const int bm = (1 << mg.lp_bits) - 1;
+                sl.run_lp = (int)interleave16((uint32_t)(key & bm), (uint32_t)((key >> g.order) & bm));
+            } else {
+                sl.run_lp = key & ((1 << mg.sm_shift) - 1);
+            }
+            sl.run_loc = sl.c_loc;
+            return;
+        }
+    }
+#endif
+    const P pix = key_to_pix<NEST, WIDE>(key, g);
+    P sm;
+    if (mg.sm_shift >= 0) {
+        sm = pix >> mg.sm_shift;
+        sl.run_lp = pix & (P)(mg.n_pix_submap - 1);
+    } else {
+        sm = pix / (P)mg.n_pix_submap;
+        sl.run_lp = pix - sm * (P)mg.n_pix_submap;
+    }
+#ifndef TB_X_NOHIT
+    if (a.hit_submaps && sm != sl.last_sm) {
+        a.hit_submaps[sm] = 1;
+        sl.last_sm = sm;
+    }
+#endif
+#ifdef TB_X_NOG2L
+    sl.run_loc = sm;
+#else
+    sl.run_loc = __ldg(&mg.global2local[sm]);
+#endif
+}
+
+// A run ends: one fp64 red per Stokes component (nothing if the submap has no storage).  Up to
+// nside 8192 the map element index fits 32 bits (< 12 * 8192^2 pixels), so the address is one
+// IMAD + one IMAD.WIDE.U32.  With TB_FOLD the run sums are unscaled (sum of tod, of tod w/r)
+// and det_scale * cal, det_scale * eta * cal are applied here, once per run.
+template <int NNZ, bool WIDE>
+__device__ __forceinline__ void flush(const Slot<typename PixT<WIDE>::T>& sl, const FusedArgs& a) {
+    if (sl.run_loc < 0) return;
+    double* dst;
+    if constexpr (WIDE) {
+        dst = a.zmap + (sl.run_loc * a.map.n_pix_submap + sl.run_lp) * NNZ;
+    } else {
+        const unsigned idx = (unsigned)sl.run_loc * (unsigned)a.map.n_pix_submap + (unsigned)sl.run_lp;
+        dst = a.zmap + (size_t)idx * NNZ;
+    }
+#if TB_FOLD
+    atomicAdd(dst, sl.r0 * sl.s_cal);
+    if (NNZ == 3) {
+        atomicAdd(dst + 1, sl.r1 * sl.s_eta);
+        atomicAdd(dst + 2, sl.r2 * sl.s_eta);
+    }
+#else
+    atomicAdd(dst, sl.r0);
+    if (NNZ == 3) {
+        atomicAdd(dst + 1, sl.r1);
+        atomicAdd(dst + 2, sl.r2);
+    }
+#endif
+}
 
 template <typename P>
 __device__ __forceinline__ void load_slot(Slot<P>& sl, const FusedArgs& a, int64_t d, bool ok, int64_t dfallback) {
@@ -366,10 +363,8 @@ __device__ __forceinline__ void load_slot(Slot<P>& sl, const FusedArgs& a, int64
     sl.r0 = sl.r1 = sl.r2 = 0.0;
     sl.pend_key = -1;
     sl.p0 = sl.p1 = sl.p2 = 0.0;
-    sl.park_key = -1;
-    sl.q0 = sl.q1 = sl.q2 = 0.0;
     sl.px = sl.py = sl.ptt = 0.0;  // dot = 0: the item's first sample takes the full arctangent
-    sl.c_smk = -1;                 // (submap key bits are >= 0: the first flush loads)
+    sl.c_smk = -1;                 // (submap key bits are >= 0: the first run start loads)
     sl.c_loc = -1;
     sl.ok = ok;
 }
@@ -389,6 +384,7 @@ __constant__ double kIncrQ[4] = {0.63661977236758134308, -0.21220659078919378103
 
 template <int NNZ, bool HWP, typename P>
 __device__ __forceinline__ StageA stage_a(Slot<P>& sl, const double* x) {
+    constexpr bool TTOFF = TB_TTOFF && TB_INCR && sizeof(P) == 4;
     StageA o;
     o.dx = x[0] * sl.u0 + x[1] * sl.u1 + x[2] * sl.u2;
     o.dy = x[3] * sl.u0 + x[4] * sl.u1 + x[5] * sl.u2;
@@ -416,19 +412,27 @@ __device__ __forceinline__ StageA stage_a(Slot<P>& sl, const double* x) {
         const double cross = fma(sl.px, o.dy, -(sl.py * o.dx));
         const double dot = fma(sl.px, o.dx, sl.py * o.dy);
         const double inv = fast_rcp(dot * r);
-        const double t = cross * (r * inv);
-        if (__double2hiint(dot) > 0 && fabs(t) <= kIncrMax) {
+        // |cross| < kIncrMax dot  <=>  dot > 0 and |t| < kIncrMax (t = cross / dot); false at
+        // dot = 0 (no previous sample) and for steps beyond a quarter turn; one DFMA + DSETP,
+        // resolved before the reciprocal's result is needed
+        if (fma(kIncrMax, dot, -fabs(cross)) > 0.0) {
+            const double t = cross * (r * inv);
             o.invr = dot * inv;
             const double s2 = t * t;
             double q = fma(kIncrQ[3], s2, kIncrQ[2]);
             q = fma(q, s2, kIncrQ[1]);
             q = fma(q, s2, kIncrQ[0]);
             double tt = fma(t, q, sl.ptt);
-            if (__double2hiint(tt) < 0) tt += 4.0;
-            if (__double2hiint(tt) >= 0x40100000) tt -= 4.0;
+            if constexpr (!TTOFF) {
+                if (__double2hiint(tt) < 0) tt += 4.0;
+                if (__double2hiint(tt) >= 0x40100000) tt -= 4.0;
+            }
             o.tt = tt;
         } else {
-            o.tt = lon_pol_raw(o.dx, o.dy, bx, by, o.cw, o.sw, o.invr);
+            // TTOFF: the chain is carried as tt + 1 WITHOUT wrapping: it restarts here from a
+            // value in [1, 5) and drifts by at most 127 steps of (2/pi) atan(0.01) = 0.0064
+            // within an item, so it stays in (0.18, 5.82); loc2key32<NEST, true> folds it back
+            o.tt = lon_pol_raw(o.dx, o.dy, bx, by, o.cw, o.sw, o.invr) + (TTOFF ? 1.0 : 0.0);
         }
         sl.px = o.dx;
         sl.py = o.dy;
@@ -450,7 +454,7 @@ __device__ __forceinline__ StageA stage_a(Slot<P>& sl, const double* x) {
 }
 
 // The HEALPix floors and integer part (branches: equatorial belt / caps): the run key.
-template <bool NEST, bool WIDE>
+template <bool NEST, int NNZ, bool WIDE>
 __device__ __forceinline__ typename PixT<WIDE>::T stage_b(const StageA& o, bool pixelise, bool ok,
                                                          const HealpixGeom& g) {
     using P = typename PixT<WIDE>::T;
@@ -462,7 +466,7 @@ __device__ __forceinline__ typename PixT<WIDE>::T stage_b(const StageA& o, bool 
 #ifdef TB_X_NOPIX
             key = (P)((int)(o.tt * 1000.0) & 0xffff);  // ablation: no HEALPix integer/floor logic
 #else
-            key = (P)loc2key32<NEST>(g, o.dz, o.tt, o.dx, o.dy);
+            key = (P)loc2key32<NEST, TB_TTOFF && TB_INCR && NNZ == 3>(g, o.dz, o.tt, o.dx, o.dy);
 #endif
     }
     if (!ok) key = -1;
@@ -475,9 +479,15 @@ __device__ __forceinline__ typename PixT<WIDE>::T stage_b(const StageA& o, bool 
 template <int NNZ, typename P>
 __device__ __forceinline__ void set_pending(Slot<P>& sl, const StageA& o, P key, double tod) {
     sl.pend_key = key;
+#if TB_FOLD
+    sl.p0 = tod;
+    if (NNZ == 3) {
+        const double t = tod * o.invr;
+#else
     sl.p0 = tod * sl.s_cal;
     if (NNZ == 3) {
         const double t = (tod * sl.s_eta) * o.invr;
+#endif
         sl.p1 = t * o.cw;
         sl.p2 = t * o.sw;
     }
@@ -493,7 +503,7 @@ __device__ __forceinline__ void det_sample(Slot<typename PixT<WIDE>::T>& sl, con
                                            int64_t s) {
     using P = typename PixT<WIDE>::T;
     const StageA o = stage_a<NNZ, HWP, P>(sl, x);
-    const P key = stage_b<NEST, WIDE>(o, pixelise, sl.ok, g);
+    const P key = stage_b<NEST, NNZ, WIDE>(o, pixelise, sl.ok, g);
     if (DEBUG && sl.ok) {
         const int64_t off = d * a.n_samp + s;
         if (a.pixels_out) a.pixels_out[off] = key < 0 ? (int64_t)-1 : (int64_t)key_to_pix<NEST, WIDE>(key, g);
@@ -517,33 +527,12 @@ __device__ __forceinline__ void det_sample(Slot<typename PixT<WIDE>::T>& sl, con
 template <bool NEST, int NNZ, bool WIDE>
 __device__ __forceinline__ void aggregate(Slot<typename PixT<WIDE>::T>& sl, const FusedArgs& a,
                                           const HealpixGeom& g) {
-#if TB_PARK
-    // PARK mode: a run that ends is parked in registers (a few moves in the divergent branch);
-    // the map work of parked runs is done once per block for the whole warp (flush_parked), so
-    // the warp no longer executes the ~40-instruction flush path at every sample where one of
-    // its 32 lanes changes pixel.  A second run end within one block flushes the parked run.
-    if (sl.pend_key >= 0 && sl.pend_key != sl.run_key) {
-        if (sl.park_key >= 0) flush_run<NEST, NNZ, WIDE>(sl.park_key, sl.q0, sl.q1, sl.q2, a, g, sl.last_sm, sl.c_smk, sl.c_loc);
-        sl.park_key = sl.run_key;
-        sl.q0 = sl.r0;
-        sl.q1 = sl.r1;
-        sl.q2 = sl.r2;
-        sl.run_key = sl.pend_key;
-        sl.r0 = sl.r1 = sl.r2 = 0.0;
-    }
-    sl.r0 += sl.p0;
-    if (NNZ == 3) {
-        sl.r1 += sl.p1;
-        sl.r2 += sl.p2;
-    }
-    return;
-#endif
     if (sl.pend_key >= 0 && sl.pend_key != sl.run_key) {
 #ifndef TB_X_NOFLUSH
-        flush<NNZ, WIDE>(sl.run_loc, sl.run_lp, sl.r0, sl.r1, sl.r2, a);
+        flush<NNZ, WIDE>(sl, a);
 #endif
         sl.run_key = sl.pend_key;
-        sl.run_loc = start_run<NEST, WIDE>(sl.pend_key, a, g, sl.last_sm, sl.run_lp);
+        start_run<NEST, WIDE>(sl.pend_key, a, g, sl);
         sl.r0 = sl.r1 = sl.r2 = 0.0;
     }
     sl.r0 += sl.p0;
@@ -605,7 +594,6 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
                                                                          unsigned long long* __restrict__ sched,
                                                                          const __grid_constant__ TmaMaps tm) {
     static_assert(!TMA || (DPL == 1 && kBlk == 16), "the TMA path stages 32 x 16 tiles");
-    constexpr bool PAIR = TB_PAIR && TMA && !DEBUG;
     using P = typename PixT<WIDE>::T;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int lane = threadIdx.x & 31;
@@ -780,7 +768,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
 #pragma unroll
         for (int j = 0; j < DPL; ++j) {
             const int row = lane + 32 * j;
-            unsigned zm = (DEBUG || PAIR) ? (~pmask & keep) : 0u;
+            unsigned zm = DEBUG ? (~pmask & keep) : 0u;
             if (have_dflags && row < cur.nrows) {
                 const unsigned rep = dmask * 0x01010101u;
                 unsigned bits = 0u;  // bit k: sample k of the box is det-flagged
@@ -821,34 +809,6 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
         const unsigned tod_row = smem_u32(&tw.tod[p][0][0]) + row_swz;
         int k = cur.k0;
         const int k_end = cur.k0 + cur.nb;
-#if TB_PAIR
-        if constexpr (PAIR) {
-            // two samples per iteration: their branch-free fp64 parts (stage_a) are issued
-            // back to back so the scheduler interleaves two independent dependency chains;
-            // shared-flagged samples run through with no key and a zeroed tod
-            for (; k + 1 < k_end; k += 2) {
-                double x0[12], x1[12];
-#pragma unroll
-                for (int i = 0; i < ((HWP && NNZ == 3) ? 12 : 10); i += 2) {
-                    const double2 t0 = *reinterpret_cast<const double2*>(st_base + 12 * k + i);
-                    const double2 t1 = *reinterpret_cast<const double2*>(st_base + 12 * k + 12 + i);
-                    x0[i] = t0.x; x0[i + 1] = t0.y;
-                    x1[i] = t1.x; x1[i + 1] = t1.y;
-                }
-                double tod0, tod1;
-                asm volatile("ld.shared.f64 %0, [%1];" : "=d"(tod0) : "r"(tod_row ^ ((unsigned)k << 3)));
-                asm volatile("ld.shared.f64 %0, [%1];" : "=d"(tod1) : "r"(tod_row ^ ((unsigned)(k + 1) << 3)));
-                const StageA o0 = stage_a<NNZ, HWP, P>(sl[0], x0);
-                const StageA o1 = stage_a<NNZ, HWP, P>(sl[0], x1);
-                aggregate<NEST, NNZ, WIDE>(sl[0], a, g);
-                const P key0 = stage_b<NEST, WIDE>(o0, (pmask >> k) & 1u, sl[0].ok, g);
-                set_pending<NNZ, P>(sl[0], o0, key0, tod0);
-                aggregate<NEST, NNZ, WIDE>(sl[0], a, g);
-                const P key1 = stage_b<NEST, WIDE>(o1, (pmask >> (k + 1)) & 1u, sl[0].ok, g);
-                set_pending<NNZ, P>(sl[0], o1, key1, tod1);
-            }
-        }
-#endif
         unsigned bit = 1u << k;  // 1 << k
 #pragma unroll kKUnroll
         for (; k < k_end; ++k, bit <<= 1) {
@@ -878,32 +838,12 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
                                                         cur.s0 + k);
         }
 
-#if TB_PARK
-        // block end: the parked runs of the whole warp in one pass
-#pragma unroll
-        for (int j = 0; j < DPL; ++j) {
-            if (sl[j].park_key >= 0) {
-                flush_run<NEST, NNZ, WIDE>(sl[j].park_key, sl[j].q0, sl[j].q1, sl[j].q2, a, g, sl[j].last_sm, sl[j].c_smk, sl[j].c_loc);
-                sl[j].park_key = -1;
-            }
-        }
         if (nxt.item != cur.item) {
 #pragma unroll
             for (int j = 0; j < DPL; ++j) {
                 aggregate<NEST, NNZ, WIDE>(sl[j], a, g);
-                if (sl[j].park_key >= 0)
-                    flush_run<NEST, NNZ, WIDE>(sl[j].park_key, sl[j].q0, sl[j].q1, sl[j].q2, a, g, sl[j].last_sm, sl[j].c_smk, sl[j].c_loc);
-                if (sl[j].run_key >= 0)
-                    flush_run<NEST, NNZ, WIDE>(sl[j].run_key, sl[j].r0, sl[j].r1, sl[j].r2, a, g, sl[j].last_sm, sl[j].c_smk, sl[j].c_loc);
+                flush<NNZ, WIDE>(sl[j], a);
             }
-#else
-        if (nxt.item != cur.item) {
-#pragma unroll
-            for (int j = 0; j < DPL; ++j) {
-                aggregate<NEST, NNZ, WIDE>(sl[j], a, g);
-                flush<NNZ, WIDE>(sl[j].run_loc, sl[j].run_lp, sl[j].r0, sl[j].r1, sl[j].r2, a);
-            }
-#endif
             if (nxt.item < 0) break;
 #pragma unroll
             for (int j = 0; j < DPL; ++j)
@@ -1316,7 +1256,7 @@ cudaError_t launch_pointing_to_tod(const WorkList& wl, const FusedArgs& a, unsig
 
 const char* last_fused_path() { return t_fused_path; }
 
-// The submap fast path of flush_run (MapGeom::sm_fast) for 32-bit keys.
+// The submap fast path of start_run (MapGeom::sm_fast) for 32-bit keys.
 FusedArgs with_submap_keys(FusedArgs a) {
     MapGeom& m = a.map;
     m.sm_fast = 0;

@@ -8,6 +8,13 @@ with detectors and observations spread over processes).
     hits = union_hit_submaps(hit_submaps)     # all_reduce(MAX) of the hit flags (tiny)
     reduce_map(zmap, hit_submaps=hits)        # pack hit submaps -> all_reduce(SUM) -> unpack
 
+Sparse, distributed map domain:
+
+    g2l, n_hit = compact_global2local(hits)   # storage for hit submaps only (-1 elsewhere)
+    own = MapOwnership.make(n_hit, world)     # contiguous blocks of hit submaps per rank
+    zc = alloc_compact_map(own, nps, nnz, dev)  # toast_pointing_to_map(..., g2l, zmap=zc)
+    block, _ = reduce_scatter_map(zc, own)    # this rank's owned, fully summed submaps
+
 Packing to the union of hit submaps shrinks the all-reduce to the sky actually observed
 (the dense map is 4.8 GB at nside 4096); the pack/unpack are index_select / index_copy on the
 device (memory plumbing, not method arithmetic).
@@ -93,3 +100,99 @@ def reduce_map(zmap: torch.Tensor, group=None, hit_submaps: Optional[torch.Tenso
     dist.all_reduce(packed, op=dist.ReduceOp.SUM, group=group)
     zmap.index_copy_(0, idx, packed)
     return zmap, packed.numel() * packed.element_size()
+
+
+# ----------------------------------------------------------------------------- sparse map domain
+# the map is stored for hit submaps only (TOAST's pixel distribution: a
+# global2local table with -1 for submaps without local storage, "accumulate ...
+# onto a sky map"), and after accumulation each rank OWNS a contiguous block of the hit
+# submaps: reduce_scatter instead of all_reduce halves the bytes each rank sends and leaves the
+# map distributed, as TOAST's distributed map domain does.  On NCCL over NVSwitch the
+# collective runs in the switch (NVLS) when NCCL enables it; there is no second implementation.
+
+def compact_global2local(hit_submaps: torch.Tensor) -> Tuple[torch.Tensor, int]:
+    """global2local of a hit-submap-only map: hit submaps get storage 0..n_hit-1 in global
+    order, the others -1 (the fused kernel skips their samples' map update — only samples in
+    unhit submaps, i.e. none, when hit_submaps is the union over ranks).  Returns (g2l int64,
+    n_hit)."""
+    hit = hit_submaps.to(torch.bool)
+    g2l = torch.full(hit.shape, -1, dtype=torch.int64, device=hit_submaps.device)
+    idx = torch.nonzero(hit, as_tuple=False).flatten()
+    g2l[idx] = torch.arange(idx.numel(), dtype=torch.int64, device=hit_submaps.device)
+    return g2l, int(idx.numel())
+
+
+@dataclasses.dataclass(frozen=True)
+class MapOwnership:
+    """Which rank owns which compact submaps after reduce_scatter_map: rank r owns compact
+    indices [r * per_rank, min(n_hit, (r + 1) * per_rank)); the compact map is padded to
+    world * per_rank submaps so every rank's block has the same size (NCCL reduce_scatter)."""
+    n_hit: int
+    world: int
+    per_rank: int
+
+    @classmethod
+    def make(cls, n_hit: int, world: int) -> "MapOwnership":
+        return cls(n_hit, world, max(1, -(-n_hit // world)))
+
+    @property
+    def padded(self) -> int:
+        return self.per_rank * self.world
+
+    def owned(self, rank: int) -> Tuple[int, int]:
+        lo = min(self.n_hit, rank * self.per_rank)
+        return lo, min(self.n_hit, lo + self.per_rank)
+
+    def owner(self, compact_index: int) -> int:
+        return compact_index // self.per_rank
+
+
+def alloc_compact_map(own: MapOwnership, n_pix_submap: int, nnz: int, device, dtype=torch.float64) -> torch.Tensor:
+    """A compact map [padded][n_pix_submap][nnz]: compact_global2local indexes its first n_hit
+    submaps; the padding submaps are never written (no global submap maps to them)."""
+    return torch.zeros((own.padded, n_pix_submap, nnz), dtype=dtype, device=device)
+
+
+def _reduce_scatter(out: torch.Tensor, inp: torch.Tensor, group=None):
+    if dist.get_backend(group) == "nccl":
+        dist.reduce_scatter_tensor(out, inp, op=dist.ReduceOp.SUM, group=group)
+    else:  # gloo has no reduce_scatter: the same result through all_reduce + this rank's slice
+        tmp = inp.clone()
+        dist.all_reduce(tmp, op=dist.ReduceOp.SUM, group=group)
+        r = dist.get_rank(group)
+        out.copy_(tmp.narrow(0, r * out.shape[0], out.shape[0]))
+
+
+def reduce_scatter_map(zmap_compact: torch.Tensor, own: MapOwnership, group=None) -> Tuple[torch.Tensor, int]:
+    """Sum the per-rank compact partial maps; return THIS rank's owned block
+    [per_rank][n_pix_submap][nnz] (rows past n_hit are padding) and the bytes each rank
+    contributes to the collective."""
+    assert zmap_compact.shape[0] == own.padded, (zmap_compact.shape, own)
+    out = torch.empty((own.per_rank,) + tuple(zmap_compact.shape[1:]), dtype=zmap_compact.dtype,
+                      device=zmap_compact.device)
+    if not (dist.is_initialized() and dist.get_world_size(group) > 1):
+        out.copy_(zmap_compact[:own.per_rank])
+        return out, 0
+    _reduce_scatter(out, zmap_compact.contiguous(), group)
+    return out, zmap_compact.numel() * zmap_compact.element_size()
+
+
+def gather_map(owned: torch.Tensor, own: MapOwnership, global2local: torch.Tensor, n_submap: int,
+               group=None) -> torch.Tensor:
+    """Reassemble the full dense map [n_submap][n_pix_submap][nnz] from the owned blocks (for
+    output; the distributed map itself never needs it).  Unhit submaps are 0."""
+    if dist.is_initialized() and dist.get_world_size(group) > 1:
+        blocks = torch.empty((own.padded,) + tuple(owned.shape[1:]), dtype=owned.dtype, device=owned.device)
+        if dist.get_backend(group) == "nccl":
+            dist.all_gather_into_tensor(blocks, owned.contiguous(), group=group)
+        else:
+            parts = [torch.empty_like(owned) for _ in range(own.world)]
+            dist.all_gather(parts, owned.contiguous(), group=group)
+            blocks = torch.cat(parts)
+    else:
+        blocks = owned
+    full = torch.zeros((n_submap,) + tuple(owned.shape[1:]), dtype=owned.dtype, device=owned.device)
+    g2l = global2local.to(owned.device)
+    hit = torch.nonzero(g2l >= 0, as_tuple=False).flatten()
+    full[hit] = blocks[g2l[hit]]
+    return full

@@ -88,3 +88,73 @@ def test_two_rank_map_reduction_equals_full_map(packed):
         np.testing.assert_array_equal(hits, href)
         assert nbytes == int(href.sum()) * w.n_pix_submap * 3 * 8
         assert nbytes < zref.nbytes
+
+
+def _worker_sparse(rank, world, port, q):
+    """f3: every rank accumulates its shard into the COMPACT (hit-submap-only) map, then
+    reduce_scatter leaves each rank its owned block; gathered, it is the oracle full map."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import oracle
+    from paper_conf_sc_demeurekktbb23_b200 import synth
+    n_det = 6
+    mine = tdist.plan_shards(tdist.make_units(1, n_det, [1], det_block=2), world)[rank]
+    full = synth.make_workload("c2", n_det=n_det, n_samp=20_000, nside=32)
+    kw = lambda w: dict(hwp=w.hwp, det_flags=w.det_flags, det_flag_mask=w.det_flag_mask,  # noqa: E731
+                        shared_flags=w.shared_flags, shared_flag_mask=w.shared_flag_mask)
+    # pass 1 (pixel distribution): hit submaps of this rank's shard from A1 -> A2 (no map)
+    hits = np.zeros(full.n_submap, np.uint8)
+    for u in mine:
+        w = synth.make_workload("c2", n_det=n_det, n_samp=20_000, nside=32, det_range=(u.d0, u.d1))
+        quats = oracle.pointing_detector(w.fp_quats, w.boresight, w.intervals, w.shared_flags, w.shared_flag_mask)
+        oracle.pixels_healpix(quats, w.intervals, w.nside, w.nest, w.n_pix_submap, w.shared_flags, w.shared_flag_mask,
+                              hit_submaps=hits)
+    ht = tdist.union_hit_submaps(torch.from_numpy(hits))
+    g2l, n_hit = tdist.compact_global2local(ht)
+    own = tdist.MapOwnership.make(n_hit, world)
+    zc = tdist.alloc_compact_map(own, full.n_pix_submap, 3, "cpu")
+    z_np = zc.numpy()
+    for u in mine:
+        w = synth.make_workload("c2", n_det=n_det, n_samp=20_000, nside=32, det_range=(u.d0, u.d1))
+        oracle.pointing_to_map(w.fp_quats, w.boresight, w.epsilon, w.cal, w.det_scale, w.det_data, w.intervals,
+                               w.nside, w.nest, 3, g2l.numpy(), w.n_pix_submap, zmap=z_np, **kw(w))
+    block, nbytes = tdist.reduce_scatter_map(zc, own)
+    lo, hi = own.owned(rank)
+    assert block.shape[0] == own.per_rank and hi - lo <= own.per_rank
+    full_map = tdist.gather_map(block, own, g2l, full.n_submap)
+    q.put((rank, full_map.numpy().copy(), ht.numpy().copy(), n_hit, lo, hi, block.numpy().copy()))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_two_rank_sparse_map_domain_reduce_scatter():
+    import oracle
+    from paper_conf_sc_demeurekktbb23_b200 import synth
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_sparse, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = sorted((q.get(timeout=120) for _ in range(2)), key=lambda r: r[0])
+    for p in procs:
+        p.join(timeout=300)
+        assert p.exitcode == 0
+    w = synth.make_workload("c2", n_det=6, n_samp=20_000, nside=32)
+    zref = np.zeros((w.n_submap, w.n_pix_submap, 3)); absmap = np.zeros_like(zref)
+    href = np.zeros(w.n_submap, np.uint8)
+    oracle.pointing_to_map(w.fp_quats, w.boresight, w.epsilon, w.cal, w.det_scale, w.det_data, w.intervals, w.nside,
+                           w.nest, 3, w.global2local, w.n_pix_submap, zmap=zref, hwp=w.hwp, det_flags=w.det_flags,
+                           det_flag_mask=w.det_flag_mask, shared_flags=w.shared_flags,
+                           shared_flag_mask=w.shared_flag_mask, hit_submaps=href, absmap=absmap)
+    from parity import check_map
+    n_hit = int(href.sum())
+    assert 0 < n_hit < w.n_submap  # the sparse domain is actually smaller than the sky
+    hit_idx = np.nonzero(href)[0]
+    for rank, full_map, hits, nh, lo, hi, block in res:
+        np.testing.assert_array_equal(hits, href)
+        assert nh == n_hit
+        check_map(full_map, zref, absmap)
+        # the owned block holds exactly this rank's slice of the hit submaps, fully summed
+        check_map(block[:hi - lo], zref[hit_idx[lo:hi]], absmap[hit_idx[lo:hi]])
+    assert res[0][5] == res[1][4]  # the two blocks tile the hit submaps
