@@ -263,7 +263,7 @@ struct Slot {
 // submap.  Sets sl.run_loc (-1: the submap has no storage) and sl.run_lp.
 template <bool NEST, bool WIDE>
 __device__ __forceinline__ void start_run(typename PixT<WIDE>::T key, const FusedArgs& a, const HealpixGeom& g,
-                                          Slot<typename PixT<WIDE>::T>& sl) {
+                                          Slot<typename PixT<WIDE>::T>& sl, uint8_t* s_hits) {
     using P = typename PixT<WIDE>::T;
     const MapGeom& mg = a.map;
 #if TB_SMCACHE
@@ -299,7 +299,9 @@ __device__ __forceinline__ void start_run(typename PixT<WIDE>::T key, const Fuse
         sl.run_lp = pix - sm * (P)mg.n_pix_submap;
     }
 #ifndef TB_X_NOHIT
-    if (a.hit_submaps && sm != sl.last_sm) {
+    if (mg.shared_hits) {
+        s_hits[sm] = 1;  // the CTA's shared copy (idempotent store, no atomic; see the kernel end)
+    } else if (a.hit_submaps && sm != sl.last_sm) {
         a.hit_submaps[sm] = 1;
         sl.last_sm = sm;
     }
@@ -526,13 +528,13 @@ __device__ __forceinline__ void det_sample(Slot<typename PixT<WIDE>::T>& sl, con
 // run of an item flushes nothing: run_loc starts at -1.
 template <bool NEST, int NNZ, bool WIDE>
 __device__ __forceinline__ void aggregate(Slot<typename PixT<WIDE>::T>& sl, const FusedArgs& a,
-                                          const HealpixGeom& g) {
+                                          const HealpixGeom& g, uint8_t* s_hits) {
     if (sl.pend_key >= 0 && sl.pend_key != sl.run_key) {
 #ifndef TB_X_NOFLUSH
         flush<NNZ, WIDE>(sl, a);
 #endif
         sl.run_key = sl.pend_key;
-        start_run<NEST, WIDE>(sl.pend_key, a, g, sl);
+        start_run<NEST, WIDE>(sl.pend_key, a, g, sl, s_hits);
         sl.r0 = sl.r1 = sl.r2 = 0.0;
     }
     sl.r0 += sl.p0;
@@ -604,6 +606,13 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
     // the alignment that matters for TMA and the swizzle is that of the shared-window offset)
     const unsigned pad1k = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
     TmaWarpSmem& tw = reinterpret_cast<TmaWarpSmem*>(smem_raw + pad1k)[wid];
+    // the CTA's hit-submap flags (MapGeom::shared_hits): after every warp's staging area
+    uint8_t* s_hits = smem_raw + (TMA ? 1024 + kWarps * sizeof(TmaWarpSmem) : kWarps * sizeof(WarpSmem<DPL>));
+    const bool shared_hits = a.map.shared_hits;
+    if (shared_hits) {
+        for (int i = threadIdx.x; i < (int)a.map.n_submap; i += blockDim.x) s_hits[i] = 0;
+        __syncthreads();
+    }
     constexpr int kRows = 32 * DPL;
     const int64_t n_groups = (a.n_det + kRows - 1) / kRows;
     const int64_t n_items = n_chunks * n_groups;
@@ -690,170 +699,177 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
     }
     prefetch_item();
     Blk cur = take_item();
-    if (cur.item < 0) return;
-    prefetch_item();
-    issue(0, cur);
-    Slot<P> sl[DPL];
+    // every thread reaches the shared-hits flush below (a warp without work skips the stream)
+    if (cur.item >= 0) [&] {
+        prefetch_item();
+        issue(0, cur);
+        Slot<P> sl[DPL];
 #pragma unroll
-    for (int j = 0; j < DPL; ++j) load_slot<P>(sl[j], a, cur.d0 + lane + 32 * j, lane + 32 * j < cur.nrows, cur.d0);
-    int p = 0;
+        for (int j = 0; j < DPL; ++j) load_slot<P>(sl[j], a, cur.d0 + lane + 32 * j, lane + 32 * j < cur.nrows, cur.d0);
+        int p = 0;
 
-    while (true) {
-        // successor block: next 16 samples of this item, or the first block of the next item
-        Blk nxt;
-        if (cur.s0 + kBlk < cur.s_end) {
-            nxt = cur;
-            nxt.s0 = cur.s0 + kBlk;
-            nxt.k0 = 0;
-            nxt.nb = (nxt.s_end - nxt.s0) < kBlk ? (int)(nxt.s_end - nxt.s0) : kBlk;
-        } else {
-            nxt = take_item();
-            if (nxt.item >= 0) prefetch_item();
-        }
-        if constexpr (TMA) {
-            mbar_wait(&tw.sf[p].mbar, (phase >> p) & 1u);
-            phase ^= 1u << p;
-        } else {
-            cp_async_wait_all();
-            __syncwarp();
-        }
-        if (nxt.item >= 0) issue(p ^ 1, nxt);
-        __syncwarp();  // reconverge after the lane-0 / spin-wait paths (else the state code below runs twice)
+        while (true) {
+            // successor block: next 16 samples of this item, or the first block of the next item
+            Blk nxt;
+            if (cur.s0 + kBlk < cur.s_end) {
+                nxt = cur;
+                nxt.s0 = cur.s0 + kBlk;
+                nxt.k0 = 0;
+                nxt.nb = (nxt.s_end - nxt.s0) < kBlk ? (int)(nxt.s_end - nxt.s0) : kBlk;
+            } else {
+                nxt = take_item();
+                if (nxt.item >= 0) prefetch_item();
+            }
+            if constexpr (TMA) {
+                mbar_wait(&tw.sf[p].mbar, (phase >> p) & 1u);
+                phase ^= 1u << p;
+            } else {
+                cp_async_wait_all();
+                __syncwarp();
+            }
+            if (nxt.item >= 0) issue(p ^ 1, nxt);
+            __syncwarp();  // reconverge after the lane-0 / spin-wait paths (else the state code below runs twice)
 
-        RawBlock<DPL>& rb = sm.buf[p];
-        // Per-sample state, split over the warp: lanes 0..kBlk-1 build the boresight rotation
-        // matrix of sample `lane` (identity if shared-flagged, S2), lanes 16..16+kBlk-1 the HWP
-        // cos/sin(4 chi) of sample `lane - 16`.  Bit k of pmask = sample k is pixelised.
-        double* st_base = TMA ? &tw.st[0][0] : &sm.st[0].v[0];
-        bool pixelise_me = false;
-        {
-            const int ks = lane & 15;
-            const bool in_blk = ks < kBlk && ks >= cur.k0 && ks < cur.k0 + cur.nb;
-            if (lane < kBlk) {
-                double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 1.0;
-                if (in_blk) {
-                    bool flagged;
+            RawBlock<DPL>& rb = sm.buf[p];
+            // Per-sample state, split over the warp: lanes 0..kBlk-1 build the boresight rotation
+            // matrix of sample `lane` (identity if shared-flagged, S2), lanes 16..16+kBlk-1 the HWP
+            // cos/sin(4 chi) of sample `lane - 16`.  Bit k of pmask = sample k is pixelised.
+            double* st_base = TMA ? &tw.st[0][0] : &sm.st[0].v[0];
+            bool pixelise_me = false;
+            {
+                const int ks = lane & 15;
+                const bool in_blk = ks < kBlk && ks >= cur.k0 && ks < cur.k0 + cur.nb;
+                if (lane < kBlk) {
+                    double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 1.0;
+                    if (in_blk) {
+                        bool flagged;
+                        if constexpr (TMA) {
+                            flagged = have_sflags && (tw.sf[p].f[lane] & smask);
+                        } else {
+                            const int soff =
+                                have_sflags ? (int)(reinterpret_cast<uintptr_t>(a.shared_flags + cur.s0) & 3) : 0;
+                            flagged = have_sflags && (rb.sflg[soff + lane] & smask);
+                        }
+                        pixelise_me = !flagged;
+                        const double* bq = TMA ? tw.bore[p][lane] : rb.bore[lane];
+                        if (!flagged) {
+                            q0 = bq[0]; q1 = bq[1]; q2 = bq[2]; q3 = bq[3];
+                        }
+                    }
+                    double m[10];
+                    quat_to_matrix(q0, q1, q2, q3, m);
+                    m[9] = 1.0;
+                    double2* dst = reinterpret_cast<double2*>(st_base + 12 * lane);
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) dst[i] = make_double2(m[2 * i], m[2 * i + 1]);
+                    st_base[12 * lane + 8] = m[8];
+                } else if (HWP && NNZ == 3 && ks < kBlk) {
+                    double c4 = 1.0, s4 = 0.0;
+                    if (in_blk) small_sincos(4.0 * (TMA ? tw.hwp[p][ks] : rb.hwp[ks]), &s4, &c4);
+                    st_base[12 * ks + 9] = c4;
+                    st_base[12 * ks + 10] = s4;
+                }
+            }
+            const unsigned pmask = __ballot_sync(0xffffffffu, pixelise_me);
+            const unsigned keep = ((1u << cur.nb) - 1u) << cur.k0;  // samples of the block processed (nb <= 16)
+            // The staged TOD of det-flagged samples (and, with debug outputs, of shared-flagged
+            // samples, which run through det_sample without a pixel) is zeroed in shared memory, so
+            // the per-sample loop needs no flag test: those samples add exactly 0 to the map.
+#pragma unroll
+            for (int j = 0; j < DPL; ++j) {
+                const int row = lane + 32 * j;
+                unsigned zm = DEBUG ? (~pmask & keep) : 0u;
+                if (have_dflags && row < cur.nrows) {
+                    const unsigned rep = dmask * 0x01010101u;
+                    unsigned bits = 0u;  // bit k: sample k of the box is det-flagged
                     if constexpr (TMA) {
-                        flagged = have_sflags && (tw.sf[p].f[lane] & smask);
+                        const uint4 f = *reinterpret_cast<const uint4*>(tw.flg[p][row]);
+                        const unsigned fw[4] = {f.x, f.y, f.z, f.w};
+#pragma unroll
+                        for (int w = 0; w < 4; ++w) {
+                            const unsigned v = __vcmpne4(fw[w] & rep, 0u);
+                            bits |= ((v & 0x01010101u) * 0x01020408u >> 24 & 0xfu) << (4 * w);
+                        }
                     } else {
-                        const int soff =
-                            have_sflags ? (int)(reinterpret_cast<uintptr_t>(a.shared_flags + cur.s0) & 3) : 0;
-                        flagged = have_sflags && (rb.sflg[soff + lane] & smask);
+                        const int foff =
+                            (int)(reinterpret_cast<uintptr_t>(a.det_flags + (cur.d0 + row) * a.n_samp + cur.s0) & 3);
+#pragma unroll
+                        for (int w = 0; w < 5; ++w) {  // bit b: byte b of the 20-byte window is flagged
+                            const unsigned v = __vcmpne4(*reinterpret_cast<const unsigned*>(&rb.flg[row][4 * w]) & rep, 0u);
+                            bits |= ((v & 0x01010101u) * 0x01020408u >> 24 & 0xfu) << (4 * w);
+                        }
+                        bits >>= foff;
                     }
-                    pixelise_me = !flagged;
-                    const double* bq = TMA ? tw.bore[p][lane] : rb.bore[lane];
-                    if (!flagged) {
-                        q0 = bq[0]; q1 = bq[1]; q2 = bq[2]; q3 = bq[3];
-                    }
+                    zm |= bits & keep;
                 }
-                double m[10];
-                quat_to_matrix(q0, q1, q2, q3, m);
-                m[9] = 1.0;
-                double2* dst = reinterpret_cast<double2*>(st_base + 12 * lane);
-#pragma unroll
-                for (int i = 0; i < 4; ++i) dst[i] = make_double2(m[2 * i], m[2 * i + 1]);
-                st_base[12 * lane + 8] = m[8];
-            } else if (HWP && NNZ == 3 && ks < kBlk) {
-                double c4 = 1.0, s4 = 0.0;
-                if (in_blk) small_sincos(4.0 * (TMA ? tw.hwp[p][ks] : rb.hwp[ks]), &s4, &c4);
-                st_base[12 * ks + 9] = c4;
-                st_base[12 * ks + 10] = s4;
-            }
-        }
-        const unsigned pmask = __ballot_sync(0xffffffffu, pixelise_me);
-        const unsigned keep = ((1u << cur.nb) - 1u) << cur.k0;  // samples of the block processed (nb <= 16)
-        // The staged TOD of det-flagged samples (and, with debug outputs, of shared-flagged
-        // samples, which run through det_sample without a pixel) is zeroed in shared memory, so
-        // the per-sample loop needs no flag test: those samples add exactly 0 to the map.
-#pragma unroll
-        for (int j = 0; j < DPL; ++j) {
-            const int row = lane + 32 * j;
-            unsigned zm = DEBUG ? (~pmask & keep) : 0u;
-            if (have_dflags && row < cur.nrows) {
-                const unsigned rep = dmask * 0x01010101u;
-                unsigned bits = 0u;  // bit k: sample k of the box is det-flagged
-                if constexpr (TMA) {
-                    const uint4 f = *reinterpret_cast<const uint4*>(tw.flg[p][row]);
-                    const unsigned fw[4] = {f.x, f.y, f.z, f.w};
-#pragma unroll
-                    for (int w = 0; w < 4; ++w) {
-                        const unsigned v = __vcmpne4(fw[w] & rep, 0u);
-                        bits |= ((v & 0x01010101u) * 0x01020408u >> 24 & 0xfu) << (4 * w);
-                    }
-                } else {
-                    const int foff =
-                        (int)(reinterpret_cast<uintptr_t>(a.det_flags + (cur.d0 + row) * a.n_samp + cur.s0) & 3);
-#pragma unroll
-                    for (int w = 0; w < 5; ++w) {  // bit b: byte b of the 20-byte window is flagged
-                        const unsigned v = __vcmpne4(*reinterpret_cast<const unsigned*>(&rb.flg[row][4 * w]) & rep, 0u);
-                        bits |= ((v & 0x01010101u) * 0x01020408u >> 24 & 0xfu) << (4 * w);
-                    }
-                    bits >>= foff;
+                while (zm) {
+                    const int k = __ffs(zm) - 1;
+                    zm &= zm - 1;
+                    if constexpr (TMA)
+                        *reinterpret_cast<double*>(reinterpret_cast<unsigned char*>(&tw.tod[p][0][0]) +
+                                                   (row_swz ^ ((unsigned)k << 3))) = 0.0;
+                    else
+                        rb.tod[row][k] = 0.0;
                 }
-                zm |= bits & keep;
             }
-            while (zm) {
-                const int k = __ffs(zm) - 1;
-                zm &= zm - 1;
-                if constexpr (TMA)
-                    *reinterpret_cast<double*>(reinterpret_cast<unsigned char*>(&tw.tod[p][0][0]) +
-                                               (row_swz ^ ((unsigned)k << 3))) = 0.0;
-                else
-                    rb.tod[row][k] = 0.0;
-            }
-        }
-        __syncwarp();
+            __syncwarp();
 
-        // TMA tile: the tile is 1 KB-aligned and row r starts at r * 128, so the swizzled address
-        // of (lane, k) is (tile + row_swz) ^ (8 k): one LOP3 per sample.
-        const unsigned tod_row = smem_u32(&tw.tod[p][0][0]) + row_swz;
-        int k = cur.k0;
-        const int k_end = cur.k0 + cur.nb;
-        unsigned bit = 1u << k;  // 1 << k
+            // TMA tile: the tile is 1 KB-aligned and row r starts at r * 128, so the swizzled address
+            // of (lane, k) is (tile + row_swz) ^ (8 k): one LOP3 per sample.
+            const unsigned tod_row = smem_u32(&tw.tod[p][0][0]) + row_swz;
+            int k = cur.k0;
+            const int k_end = cur.k0 + cur.nb;
+            unsigned bit = 1u << k;  // 1 << k
 #pragma unroll kKUnroll
-        for (; k < k_end; ++k, bit <<= 1) {
-            const bool pixelise = pmask & bit;
-            if (!DEBUG && !pixelise) continue;  // shared-flagged sample: nothing to add (uniform)
-            double x[12];
+            for (; k < k_end; ++k, bit <<= 1) {
+                const bool pixelise = pmask & bit;
+                if (!DEBUG && !pixelise) continue;  // shared-flagged sample: nothing to add (uniform)
+                double x[12];
 #pragma unroll
-            for (int i = 0; i < ((HWP && NNZ == 3) ? 12 : 10); i += 2) {
-                const double2 t2 = *reinterpret_cast<const double2*>(st_base + 12 * k + i);
-                x[i] = t2.x;
-                x[i + 1] = t2.y;
+                for (int i = 0; i < ((HWP && NNZ == 3) ? 12 : 10); i += 2) {
+                    const double2 t2 = *reinterpret_cast<const double2*>(st_base + 12 * k + i);
+                    x[i] = t2.x;
+                    x[i + 1] = t2.y;
+                }
+                double tod[DPL];
+#pragma unroll
+                for (int j = 0; j < DPL; ++j) {
+                    if constexpr (TMA)
+                        asm volatile("ld.shared.f64 %0, [%1];" : "=d"(tod[j]) : "r"(tod_row ^ ((unsigned)k << 3)));
+                    else
+                        tod[j] = rb.tod[lane + 32 * j][k];
+                }
+                // fold the previous sample while those shared-memory loads are in flight
+#pragma unroll
+                for (int j = 0; j < DPL; ++j) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, s_hits);
+#pragma unroll
+                for (int j = 0; j < DPL; ++j)
+                    det_sample<NEST, NNZ, HWP, DEBUG, WIDE>(sl[j], x, pixelise, tod[j], g, a, cur.d0 + lane + 32 * j,
+                                                            cur.s0 + k);
             }
-            double tod[DPL];
-#pragma unroll
-            for (int j = 0; j < DPL; ++j) {
-                if constexpr (TMA)
-                    asm volatile("ld.shared.f64 %0, [%1];" : "=d"(tod[j]) : "r"(tod_row ^ ((unsigned)k << 3)));
-                else
-                    tod[j] = rb.tod[lane + 32 * j][k];
-            }
-            // fold the previous sample while those shared-memory loads are in flight
-#pragma unroll
-            for (int j = 0; j < DPL; ++j) aggregate<NEST, NNZ, WIDE>(sl[j], a, g);
-#pragma unroll
-            for (int j = 0; j < DPL; ++j)
-                det_sample<NEST, NNZ, HWP, DEBUG, WIDE>(sl[j], x, pixelise, tod[j], g, a, cur.d0 + lane + 32 * j,
-                                                        cur.s0 + k);
-        }
 
-        if (nxt.item != cur.item) {
+            if (nxt.item != cur.item) {
 #pragma unroll
-            for (int j = 0; j < DPL; ++j) {
-                aggregate<NEST, NNZ, WIDE>(sl[j], a, g);
-                flush<NNZ, WIDE>(sl[j], a);
+                for (int j = 0; j < DPL; ++j) {
+                    aggregate<NEST, NNZ, WIDE>(sl[j], a, g, s_hits);
+                    flush<NNZ, WIDE>(sl[j], a);
+                }
+                if (nxt.item < 0) break;
+#pragma unroll
+                for (int j = 0; j < DPL; ++j)
+                    load_slot<P>(sl[j], a, nxt.d0 + lane + 32 * j, lane + 32 * j < nxt.nrows, nxt.d0);
             }
-            if (nxt.item < 0) break;
-#pragma unroll
-            for (int j = 0; j < DPL; ++j)
-                load_slot<P>(sl[j], a, nxt.d0 + lane + 32 * j, lane + 32 * j < nxt.nrows, nxt.d0);
+            __syncwarp();  // all lanes are done with buffer p and st before they are refilled
+            cur = nxt;
+            p ^= 1;
         }
-        __syncwarp();  // all lanes are done with buffer p and st before they are refilled
-        cur = nxt;
-        p ^= 1;
+        if constexpr (!TMA) cp_async_wait_all();
+    }();
+    if (shared_hits) {  // the CTA's hit flags, once: a few hundred stores instead of one per run
+        __syncthreads();
+        for (int i = threadIdx.x; i < (int)a.map.n_submap; i += blockDim.x)
+            if (s_hits[i]) a.hit_submaps[i] = 1;
     }
-    if constexpr (!TMA) cp_async_wait_all();
 }
 
 // Tensor-map encoder from the driver, fetched through the runtime (no link against libcuda).
@@ -950,7 +966,8 @@ template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL, bool TMA
 cudaError_t launch_k(const WorkList& wl, const FusedArgs& a, const TmaMaps& tm, unsigned long long* sched,
                      cudaStream_t st) {
     auto kern = pointing_to_map_kernel<NEST, NNZ, HWP, DEBUG, WIDE, DPL, TMA>;
-    const size_t smem = TMA ? sizeof(TmaWarpSmem) * kWarps + 1024 : sizeof(WarpSmem<DPL>) * kWarps;
+    const size_t smem =
+        (TMA ? sizeof(TmaWarpSmem) * kWarps + 1024 : sizeof(WarpSmem<DPL>) * kWarps) + kSharedHitBytes;
     static int blocks_per_sm = 0;
     static std::once_flag once;
     std::call_once(once, [&] {
@@ -1259,6 +1276,8 @@ const char* last_fused_path() { return t_fused_path; }
 // The submap fast path of start_run (MapGeom::sm_fast) for 32-bit keys.
 FusedArgs with_submap_keys(FusedArgs a) {
     MapGeom& m = a.map;
+    m.n_submap = (12 * a.nside * a.nside + m.n_pix_submap - 1) / m.n_pix_submap;
+    m.shared_hits = a.hit_submaps != nullptr && m.n_submap <= kSharedHitBytes;
     m.sm_fast = 0;
     if (a.nside > 8192 || m.sm_shift < 0) return a;
     int order = 0;

@@ -38,7 +38,16 @@ struct MapGeom {
     int sm_fast = 0;
     int smk_mask = 0;
     int lp_bits = 0;
+    // fused pointing_to_map only (set at launch): n_submap = 12 nside^2 / n_pix_submap, and
+    // whether the hit-submap flags are gathered in a per-CTA shared-memory copy (n_submap <=
+    // kSharedHitBytes) and written to hit_submaps once per CTA at the end.
+    int64_t n_submap = 0;
+    int shared_hits = 0;
 };
+
+// Shared-memory hit-submap flags per CTA of the fused kernel (n_submap = 3072 at every nside
+// >= 16 with the 16x16-submap layout of the benchmarks).
+constexpr int kSharedHitBytes = 8192;
 
 struct FusedArgs {
     const double* fp_quats;

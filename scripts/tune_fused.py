@@ -20,7 +20,7 @@ sys.path.insert(0, os.environ["ROOT"])
 import torch
 from paper_conf_sc_demeurekktbb23_b200 import binding, synth
 from paper_conf_sc_demeurekktbb23_b200.staging import DeviceWorkload
-w = synth.make_workload(os.environ["WL"])
+w = synth.make_workload(os.environ["WL"], **json.loads(os.environ.get("WLARGS", "{}")))
 dw = DeviceWorkload.upload(w, "cuda")
 raw = dw.raw_args()
 lib = binding.load()
@@ -45,16 +45,17 @@ print(json.dumps({"lib": os.environ.get("TOASTB200_LIB", "default"), "ms": ms,
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--workload", default="c2")
+    ap.add_argument("--wlargs", default="{}", help="JSON overrides for synth.make_workload (nside, nest, n_det, ...)")
     ap.add_argument("libs", nargs="*")
     args = ap.parse_args()
     libs = args.libs or [None]
     for lib in libs:
-        env = dict(os.environ, ROOT=ROOT, WL=args.workload)
+        env = dict(os.environ, ROOT=ROOT, WL=args.workload, WLARGS=args.wlargs)
         if lib:
             env["TOASTB200_LIB"] = os.path.abspath(lib)
         r = subprocess.run([sys.executable, "-c", CHILD], env=env, capture_output=True, text=True)
         line = r.stdout.strip().splitlines()[-1] if r.stdout.strip() else json.dumps({"lib": lib, "error": r.stderr[-800:]})
-        print(line, flush=True)
+        print(line.rstrip("}") + f', "wl": "{args.workload}", "wlargs": {args.wlargs}}}', flush=True)
 
 
 if __name__ == "__main__":
