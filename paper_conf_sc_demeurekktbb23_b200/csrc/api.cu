@@ -119,6 +119,18 @@ int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, WorkList
     return TOAST_OK;
 }
 
+// Work list of the fused kernels: chunks of kFusedChunk samples, shorter when few detector groups
+// x few samples would leave the persistent grid idle (C1: 4 detectors, one group of 32 lanes),
+// so that there are at least ~4 items per resident warp.
+int fused_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, int64_t n_det, WorkList* out) {
+    int rc = get_worklist(iv, n, n_samp, out, kFusedChunk);
+    if (rc != TOAST_OK) return rc;
+    const int64_t groups = (n_det + 31) / 32, want = 4 * (int64_t)num_sms() * 16;
+    int chunk = kFusedChunk;
+    while (chunk > 16 && (out->n_samples / chunk) * groups < want) chunk /= 2;
+    return chunk == kFusedChunk ? TOAST_OK : get_worklist(iv, n, n_samp, out, chunk);
+}
+
 bool is_pow2(int64_t x) { return x > 0 && (x & (x - 1)) == 0; }
 
 int check_nside(int64_t nside) {
@@ -371,7 +383,7 @@ int toast_pointing_to_map(const double* fp_quats, const double* boresight, const
         REQUIRE(zmap);
     }
     WorkList wl;
-    rc = get_worklist(intervals, n_intervals, n_samp, &wl, kFusedChunk);
+    rc = fused_worklist(intervals, n_intervals, n_samp, n_det, &wl);
     if (rc != TOAST_OK) return rc;
     FusedArgs a;
     a.fp_quats = fp_quats;
@@ -429,7 +441,7 @@ extern "C" int toast_pointing_to_tod(const double* fp_quats, const double* bores
         REQUIRE(det_data);
     }
     WorkList wl;
-    rc = get_worklist(intervals, n_intervals, n_samp, &wl, kFusedChunk);
+    rc = fused_worklist(intervals, n_intervals, n_samp, n_det, &wl);
     if (rc != TOAST_OK) return rc;
     FusedArgs a = {};
     a.fp_quats = fp_quats;

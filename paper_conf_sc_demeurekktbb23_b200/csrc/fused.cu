@@ -68,8 +68,8 @@ constexpr int kKUnroll = TB_KUNROLL;  // unroll of the per-sample loop
 #ifndef TB_TTOFF
 #define TB_TTOFF 1  // 32-bit keys: longitude carried as tt + 1 without wrapping (see stage_a)
 #endif
-#ifndef TB_SMCACHE
-#define TB_SMCACHE 0  // run start: per-lane submap cache (measured on B200: -1.5% C2, -0.5% C3; off)
+#ifndef TB_HITDEDUP
+#define TB_HITDEDUP 1  // shared hit flags: store only when the lane's submap changes
 #endif
 constexpr int kPad = kBlk + 1;
 
@@ -244,8 +244,6 @@ struct Slot {
     P run_lp;             // its pixel's index inside the submap
     int64_t run_loc;      // global2local of the run's submap, LOADED WHEN THE RUN STARTS
     P last_sm;            // last submap this lane marked in hit_submaps (generic path)
-    int c_smk;            // MapGeom::sm_fast: submap key bits of the last run start
-    int64_t c_loc;        //   and its global2local entry
     double r0, r1, r2;
     P pend_key;           // pending (not yet aggregated) det-sample
     double p0, p1, p2;
@@ -257,38 +255,12 @@ struct Slot {
 // the load latency is hidden behind the run's samples instead of stalling the flush.  The hit
 // flag is stored only when the lane's submap CHANGES: thousands of warps re-writing the same
 // few bytes of hit_submaps serialise in L2 and cost as much as the whole computation.
-// With MapGeom::sm_fast (32-bit keys, power-of-two submaps) the submap is read off the key bits
-// and compared with the lane's last one: a run in the same submap (nearly all of them) needs
-// neither the pixel, the hit mark nor the global2local load — only the pixel's index inside the
-// submap.  Sets sl.run_loc (-1: the submap has no storage) and sl.run_lp.
+// Sets sl.run_loc (-1: the submap has no storage) and sl.run_lp.
 template <bool NEST, bool WIDE>
 __device__ __forceinline__ void start_run(typename PixT<WIDE>::T key, const FusedArgs& a, const HealpixGeom& g,
                                           Slot<typename PixT<WIDE>::T>& sl, uint8_t* s_hits) {
     using P = typename PixT<WIDE>::T;
     const MapGeom& mg = a.map;
-#if TB_SMCACHE
-    if constexpr (!WIDE) {
-        if (mg.sm_fast) {
-            const int smk = NEST ? (key & mg.smk_mask) : (key >> mg.sm_shift);
-            if (smk != sl.c_smk) {
-                const int sm = key_to_pix<NEST, WIDE>(key, g) >> mg.sm_shift;
-#ifndef TB_X_NOHIT
-                if (a.hit_submaps) a.hit_submaps[sm] = 1;
-#endif
-                sl.c_loc = __ldg(&mg.global2local[sm]);
-                sl.c_smk = smk;
-            }
-            if (NEST) {
-                const int bm = (1 << mg.lp_bits) - 1;
-                sl.run_lp = (int)interleave16((uint32_t)(key & bm), (uint32_t)((key >> g.order) & bm));
-            } else {
-                sl.run_lp = key & ((1 << mg.sm_shift) - 1);
-            }
-            sl.run_loc = sl.c_loc;
-            return;
-        }
-    }
-#endif
     const P pix = key_to_pix<NEST, WIDE>(key, g);
     P sm;
     if (mg.sm_shift >= 0) {
@@ -300,7 +272,15 @@ __device__ __forceinline__ void start_run(typename PixT<WIDE>::T key, const Fuse
     }
 #ifndef TB_X_NOHIT
     if (mg.shared_hits) {
-        s_hits[sm] = 1;  // the CTA's shared copy (idempotent store, no atomic; see the kernel end)
+        // the CTA's shared copy (idempotent store, no atomic; see the kernel end)
+#if TB_HITDEDUP
+        if (sm != sl.last_sm) {
+            s_hits[sm] = 1;
+            sl.last_sm = sm;
+        }
+#else
+        s_hits[sm] = 1;
+#endif
     } else if (a.hit_submaps && sm != sl.last_sm) {
         a.hit_submaps[sm] = 1;
         sl.last_sm = sm;
@@ -366,8 +346,6 @@ __device__ __forceinline__ void load_slot(Slot<P>& sl, const FusedArgs& a, int64
     sl.pend_key = -1;
     sl.p0 = sl.p1 = sl.p2 = 0.0;
     sl.px = sl.py = sl.ptt = 0.0;  // dot = 0: the item's first sample takes the full arctangent
-    sl.c_smk = -1;                 // (submap key bits are >= 0: the first run start loads)
-    sl.c_loc = -1;
     sl.ok = ok;
 }
 
@@ -1273,29 +1251,18 @@ cudaError_t launch_pointing_to_tod(const WorkList& wl, const FusedArgs& a, unsig
 
 const char* last_fused_path() { return t_fused_path; }
 
-// The submap fast path of start_run (MapGeom::sm_fast) for 32-bit keys.
-FusedArgs with_submap_keys(FusedArgs a) {
+// Launch-side map geometry of the fused kernel: the submap count and whether the hit flags
+// are gathered in shared memory.
+FusedArgs with_map_geom(FusedArgs a) {
     MapGeom& m = a.map;
     m.n_submap = (12 * a.nside * a.nside + m.n_pix_submap - 1) / m.n_pix_submap;
     m.shared_hits = a.hit_submaps != nullptr && m.n_submap <= kSharedHitBytes;
-    m.sm_fast = 0;
-    if (a.nside > 8192 || m.sm_shift < 0) return a;
-    int order = 0;
-    while ((int64_t(1) << order) < a.nside) ++order;
-    if (!a.nest) {
-        m.sm_fast = 1;
-    } else if (m.sm_shift % 2 == 0 && m.sm_shift / 2 <= order) {
-        const int b = m.sm_shift / 2;
-        m.lp_bits = b;
-        m.smk_mask = ~((((1 << b) - 1) << order) | ((1 << b) - 1));
-        m.sm_fast = 1;
-    }
     return a;
 }
 
 cudaError_t launch_pointing_to_map(const WorkList& wl, const FusedArgs& a_in, unsigned long long* sched,
                                    cudaStream_t st) {
-    const FusedArgs a = with_submap_keys(a_in);
+    const FusedArgs a = with_map_geom(a_in);
     if (wl.n_chunks == 0 || a.n_det == 0) return cudaSuccess;
     if (a.nest) return a.nnz == 3 ? dispatch_hwp<true, 3>(wl, a, sched, st) : dispatch_hwp<true, 1>(wl, a, sched, st);
     return a.nnz == 3 ? dispatch_hwp<false, 3>(wl, a, sched, st) : dispatch_hwp<false, 1>(wl, a, sched, st);

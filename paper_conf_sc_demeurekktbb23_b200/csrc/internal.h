@@ -31,13 +31,6 @@ struct MapGeom {
     const int64_t* global2local;
     int64_t n_pix_submap;
     int sm_shift;         // log2(n_pix_submap) if a power of two, else -1
-    // fused kernels only (set at launch): the submap of a 32-bit run key without forming the
-    // pixel.  NEST with n_pix_submap = 4^b <= nside^2: key & smk_mask identifies the submap and
-    // the pixel inside it is the interleave of the low b bits of ix and iy; RING with a power
-    // of two n_pix_submap: key >> sm_shift.  sm_fast = 0: the generic path.
-    int sm_fast = 0;
-    int smk_mask = 0;
-    int lp_bits = 0;
     // fused pointing_to_map only (set at launch): n_submap = 12 nside^2 / n_pix_submap, and
     // whether the hit-submap flags are gathered in a per-CTA shared-memory copy (n_submap <=
     // kSharedHitBytes) and written to hit_submaps once per CTA at the end.

@@ -1,0 +1,8 @@
+bash scripts/gpu_check.sh r01m c2
+OUT=gpurun_out/r01m
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:pointing_to_map -s 4 -c 1 \
+    -o $OUT/prof_fused_c3 python bench.py --workload c3 --steps 2 --warmup 3 --soak 0 --no-e2e --no-cpu-baseline > $OUT/ncu_full_c3.log 2>&1
+for w in c1 c3 c4 c5; do timeout 900 python bench.py --workload $w --steps 10 --warmup 3 > $OUT/bench_$w.json 2> $OUT/bench_$w.err; done
+timeout 600 python bench.py --workload c5 --steps 10 --warmup 3 --no-cpu-baseline --reduce scatter > $OUT/bench_c5_compact.json 2> $OUT/bench_c5_compact.err
+timeout 600 python bench.py --impl reference --steps 3 --warmup 1 > $OUT/bench_reference.json 2> $OUT/bench_reference.err
+bash scripts/ops_check.sh r01m "c2 c3"
