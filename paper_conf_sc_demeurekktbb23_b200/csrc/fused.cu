@@ -1068,8 +1068,8 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_tod_ke
     Slot<P> sl;
     load_slot<P>(sl, a, cur.d0 + lane, lane < cur.nrows, cur.d0);
     int p = 0;
-    // per-lane gather cache: map values of pixel cur_pix (loc < 0: no storage)
-    P cur_pix = -1;
+    // per-lane gather cache: map values of the pixel of run key cur_key (loc < 0: no storage)
+    P cur_key = -1;
     int64_t cur_loc = -1, last_sm = -1, last_loc = -1;
     double m0 = 0.0, m1 = 0.0, m2 = 0.0;
 
@@ -1132,38 +1132,20 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_tod_ke
                 x[i + 1] = t2.y;
             }
             const double tod = rb.tod[lane][k];
-            const double dx = x[0] * sl.u0 + x[1] * sl.u1 + x[2] * sl.u2;
-            const double dy = x[3] * sl.u0 + x[4] * sl.u1 + x[5] * sl.u2;
-            const double dz = x[6] * sl.u0 + x[7] * sl.u1 + x[8] * sl.u2;
-            double c2 = 0.0, s2 = 0.0, tt;
-            if (NNZ == 3) {
-                const double bx = x[6] * sl.v0 + x[7] * sl.v1 + x[8] * sl.v2;
-                const double by = -(x[6] * sl.w0 + x[7] * sl.w1 + x[8] * sl.w2);
-                tt = lon_pol(dx, dy, bx, by, c2, s2);
-                if (HWP) {
-                    const double c4 = x[9], s4 = x[10];
-                    const double cq = c2 * c4 - s2 * s4;
-                    const double sq = s2 * c4 + c2 * s4;
-                    c2 = cq;
-                    s2 = sq;
-                }
-            } else {
-                tt = quarter_turns(dx, dy);
-            }
-            P pix;
-            if (WIDE)
-                pix = (P)loc2pix<NEST, int64_t>(g, dz, tt, dx, dy);
-            else
-                pix = (P)loc2pix32<NEST>(g, dz, tt, dx, dy);
-            if (!sl.ok) pix = -1;
+            // the same per-det-sample arithmetic as pointing_to_map (incremental longitude,
+            // algebraic weights, run keys): cos 2psi' = cw / r, sin 2psi' = sw / r
+            const StageA o = stage_a<NNZ, HWP, P>(sl, x);
+            const P key = stage_b<NEST, NNZ, WIDE>(o, true, sl.ok, g);
+            const double c2 = o.cw * o.invr, s2 = o.sw * o.invr;
             finish();  // the previous sample's gathered values have arrived by now
-            if (pix >= 0 && pix != cur_pix) {
+            if (key >= 0 && key != cur_key) {
+                const P pix = key_to_pix<NEST, WIDE>(key, g);
                 const int64_t smi = submap_of<P>(pix, mg);
                 if (smi != last_sm) {
                     last_loc = __ldg(&mg.global2local[smi]);
                     last_sm = smi;
                 }
-                cur_pix = pix;
+                cur_key = key;  // the run key of the cached pixel
                 cur_loc = last_loc;
                 if (cur_loc >= 0) {
                     const int64_t lp = mg.sm_shift >= 0 ? (int64_t)(pix & (P)(mg.n_pix_submap - 1))
@@ -1176,7 +1158,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_tod_ke
                     }
                 }
             }
-            if (pix >= 0 && cur_loc >= 0) {
+            if (key >= 0 && cur_loc >= 0) {
                 pend_k = k;
                 pend_tod = tod;
                 pend_c2 = c2;
@@ -1198,7 +1180,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_tod_ke
         if (nxt.item != cur.item) {
             if (nxt.item < 0) break;
             load_slot<P>(sl, a, nxt.d0 + lane, lane < nxt.nrows, nxt.d0);
-            cur_pix = -1;
+            cur_key = -1;
             cur_loc = -1;
         }
         __syncwarp();

@@ -176,6 +176,70 @@ __global__ void __launch_bounds__(kChunk) offset_project_kernel(
     }
 }
 
+// Projection for step >= kSpan (the destriper's usual steps are hundreds of samples): a WARP
+// owns one (chunk, detector) pair and lane L sums the kSpan consecutive samples
+// [8L, 8L + 8) of the chunk in registers.  With step >= kSpan a lane meets at most one step
+// boundary, so it holds two partial sums: A for its first amplitude r and B for r + 1.  B is
+// handed to the next lane (whose first amplitude is r + 1) by one shuffle, then ONE segmented
+// scan over the 32 lanes sums each amplitude and its last lane issues one fp64 red — one scan
+// per 256 samples instead of one per 32 (offset_project_kernel), the loads 8 deep per thread.
+constexpr int kSpan = 8;
+static_assert(kSpan * 32 == kChunk, "a warp covers one work chunk");
+
+template <bool IDX>
+__global__ void __launch_bounds__(kChunk) offset_project_span_kernel(
+    const Chunk* __restrict__ chunks, int64_t n_chunks, OffsetViews v, const int64_t* __restrict__ amp_offset,
+    double* __restrict__ amplitudes, const int32_t* __restrict__ data_index, const double* __restrict__ det_data,
+    const int32_t* __restrict__ flag_index, const uint8_t* __restrict__ det_flags, uint8_t det_flag_mask,
+    int64_t n_det, int64_t n_samp) {
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    constexpr int kWarpsPerCta = kChunk / 32;
+    for (int64_t c = blockIdx.x; c < n_chunks; c += gridDim.x) {
+        const Chunk ch = chunks[c];
+        const int k0 = kSpan * lane;
+        const int n = max(0, min(kSpan, ch.count - k0));  // this lane's samples in the chunk
+        const bool ok = n > 0;
+        const bool next_ok = lane < 31 && k0 + kSpan < ch.count;
+        const int64_t s0 = ch.first + k0;
+        const int off0 = (int)(s0 - __ldg(&v.iv_first[ch.interval]));
+        const int r = off0 / v.step;                // amplitude of the lane's first sample in its interval
+        const int kb = (r + 1) * v.step - off0;     // first lane-local sample of amplitude r + 1 (>= 1)
+        const int64_t base = __ldg(&v.view_base[ch.interval]);
+        const int rprev = __shfl_up_sync(kFullMask, r, 1);
+        const bool okprev = __shfl_up_sync(kFullMask, ok, 1);
+        const bool head = lane == 0 || rprev != r || !okprev || !ok;
+        const unsigned heads = __ballot_sync(kFullMask, head);
+        const int depth = lane - (31 - __clz(heads & (kFullMask >> (31 - lane))));
+        const bool tail = lane == 31 || ((heads >> (lane + 1)) & 1u);
+        for (int64_t d = (int64_t)blockIdx.y * kWarpsPerCta + warp; d < n_det; d += (int64_t)gridDim.y * kWarpsPerCta) {
+            const double* t = det_data + row_or<IDX>(data_index, d) * n_samp + s0;
+            const uint8_t* f = det_flags ? det_flags + row_or<IDX>(flag_index, d) * n_samp + s0 : nullptr;
+            double A = 0.0, B = 0.0;
+#pragma unroll
+            for (int k = 0; k < kSpan; ++k) {
+                if (k < n) {
+                    double x = __ldg(t + k);
+                    if (f && (__ldg(f + k) & det_flag_mask)) x = 0.0;
+                    if (k < kb) A += x; else B += x;
+                }
+            }
+            const int64_t a0 = ok ? __ldg(&amp_offset[d]) + base : 0;
+            const double Bp = __shfl_up_sync(kFullMask, B, 1);
+            if (lane > 0 && ok) A += Bp;  // the previous lane's tail belongs to my first amplitude
+            if (ok && kb < n && !next_ok) atomicAdd(&amplitudes[a0 + r + 1], B);  // no next lane to take it
+            double x = A;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                if (!__any_sync(kFullMask, depth >= o)) break;
+                const double y = __shfl_up_sync(kFullMask, x, o);
+                if (depth >= o) x += y;
+            }
+            if (tail && ok) atomicAdd(&amplitudes[a0 + r], x);
+        }
+    }
+}
+
 __global__ void precond_kernel(const double* __restrict__ var, const double* __restrict__ in,
                                double* __restrict__ out, int64_t n) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
@@ -214,7 +278,16 @@ cudaError_t launch_offset_project(const WorkList& wl, const OffsetViews& v, cons
                                   const int32_t* flag_index, const uint8_t* det_flags, uint8_t det_flag_mask,
                                   int64_t n_det, int64_t n_samp, cudaStream_t st) {
     if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
-    (data_index || flag_index ? offset_project_kernel<true> : offset_project_kernel<false>)<<<grid_dt(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, v, amp_offset, amplitudes,
+    const bool idx = data_index || flag_index;
+    if (v.step >= kSpan) {
+        const dim3 grid((unsigned)std::min<int64_t>(wl.n_chunks, 0x7fffffff),
+                        (unsigned)std::min<int64_t>((n_det + kChunk / 32 - 1) / (kChunk / 32), 65535), 1);
+        (idx ? offset_project_span_kernel<true> : offset_project_span_kernel<false>)<<<grid, kChunk, 0, st>>>(
+            wl.chunks, wl.n_chunks, v, amp_offset, amplitudes, data_index, det_data, flag_index, det_flags,
+            det_flag_mask, n_det, n_samp);
+        return cudaGetLastError();
+    }
+    (idx ? offset_project_kernel<true> : offset_project_kernel<false>)<<<grid_dt(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, v, amp_offset, amplitudes,
                                                                 data_index, det_data, flag_index, det_flags,
                                                                 det_flag_mask, n_det, n_samp);
     return cudaGetLastError();
