@@ -42,11 +42,12 @@ constexpr double kTanPi8 = 0.41421356237309504880;
 // Constants whose low word is non-zero are kept in the constant bank so that the fp64
 // instructions take them as c[][] operands: written as literals, the compiler re-materialises
 // them with two UMOVs per use inside the hot loop once the uniform registers run out.
-static __constant__ double kC[4] = {kTanPi8, 1e-100, 2.0 / 3.0, 0.99};
+static __constant__ double kC[5] = {kTanPi8, 1e-100, 2.0 / 3.0, 0.99, 0.01};
 #define TB_TAN_PI8 (::toastb200::kC[0])
 #define TB_TINY (::toastb200::kC[1])
 #define TB_TWO_THIRD (::toastb200::kC[2])
 #define TB_CAP_SINTHETA_Z (::toastb200::kC[3])
+#define TB_INCR_MAX (::toastb200::kC[4])  // kIncrMax of the fused kernel's incremental longitude
 
 // 1/x for finite x > 0 (no IEEE rounding guarantee; <= ~1 ulp): MUFU seed + ONE cubic step,
 // r' = r + r (e + e^2) with e = 1 - x r.  Measured on B200 (scripts/mufu_precision.cu, 2^24
@@ -441,14 +442,14 @@ __device__ __forceinline__ int loc2key32(const HealpixGeom& g, double dz, double
             const int ip = (t1 >> 1) & (nl4 - 1);
             return (int)g.ncap + nl4 * (ir - 1) + ip;
         } else {
-            int ifp = jp >> g.order;
-            int ifm = jm >> g.order;
-            int face;
-            if (OFF) {  // ifp, ifm in 0..6 stand for faces (ifp - 1) mod 4, (ifm - 1) mod 4
-                face = (ifp == ifm) ? (((ifp + 3) & 3) | 4) : ((ifp < ifm) ? ((ifp + 3) & 3) : (((ifm + 3) & 3) | 8));
-            } else {
-                face = (ifp == ifm) ? (ifp | 4) : ((ifp < ifm) ? ifp : (ifm + 8));
-            }
+            const int ifp = jp >> g.order;
+            const int ifm = jm >> g.order;
+            // face = ifp | 4 (ifp == ifm), ifp (ifp < ifm), ifm + 8 (ifp > ifm), with the face
+            // row indices taken mod 4 (ifp, ifm reach 4 at tt near 4; OFF: they run 0..6 and
+            // stand for ifp - 1, ifm - 1): |ifp - ifm| <= 1, so branch-free as
+            // (min(ifp, ifm) mod 4) + 4 (1 + ifp - ifm)
+            const int fmin = (ifp < ifm ? ifp : ifm) + (OFF ? 3 : 0);
+            const int face = (fmin & 3) + 4 * (1 + ifp - ifm);
             const int ix = jm & m;
             const int iy = (jp & m) ^ m;  // nside - 1 - (jp & (nside - 1))
             return (face * nside + iy) * nside + ix;

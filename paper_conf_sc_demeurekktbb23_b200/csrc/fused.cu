@@ -68,6 +68,9 @@ constexpr int kKUnroll = TB_KUNROLL;  // unroll of the per-sample loop
 #ifndef TB_TTOFF
 #define TB_TTOFF 1  // 32-bit keys: longitude carried as tt + 1 without wrapping (see stage_a)
 #endif
+#ifndef TB_DEFER
+#define TB_DEFER 1  // a det-sample's contribution is folded into its run one sample later
+#endif
 #ifndef TB_HITDEDUP
 #define TB_HITDEDUP 1  // shared hit flags: store only when the lane's submap changes
 #endif
@@ -356,9 +359,8 @@ struct StageA {
     double cw, sw, invr;  // r cos 2(psi + 2 chi), r sin 2(psi + 2 chi), 1/r
 };
 
-// (2/pi) atan(t) = t Q(t^2) for |t| <= kIncrMax: the Taylor series to t^7; the first omitted
-// term is (2/pi) t^9 / 9 <= 7e-20 (absolute) at |t| = 0.01.
-constexpr double kIncrMax = 0.01;
+// (2/pi) atan(t) = t Q(t^2) for |t| <= kIncrMax = 0.01 (TB_INCR_MAX, in the constant bank): the
+// Taylor series to t^7; the first omitted term is (2/pi) t^9 / 9 <= 7e-20 (absolute) at |t| = 0.01.
 __constant__ double kIncrQ[4] = {0.63661977236758134308, -0.21220659078919378103, 0.12732395447351626862,
                                  -0.090945681766797334729};
 
@@ -395,7 +397,7 @@ __device__ __forceinline__ StageA stage_a(Slot<P>& sl, const double* x) {
         // |cross| < kIncrMax dot  <=>  dot > 0 and |t| < kIncrMax (t = cross / dot); false at
         // dot = 0 (no previous sample) and for steps beyond a quarter turn; one DFMA + DSETP,
         // resolved before the reciprocal's result is needed
-        if (fma(kIncrMax, dot, -fabs(cross)) > 0.0) {
+        if (fma(TB_INCR_MAX, dot, -fabs(cross)) > 0.0) {
             const double t = cross * (r * inv);
             o.invr = dot * inv;
             const double s2 = t * t;
@@ -817,19 +819,26 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
                     else
                         tod[j] = rb.tod[lane + 32 * j][k];
                 }
+#if TB_DEFER
                 // fold the previous sample while those shared-memory loads are in flight
 #pragma unroll
                 for (int j = 0; j < DPL; ++j) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, s_hits);
+#endif
 #pragma unroll
                 for (int j = 0; j < DPL; ++j)
                     det_sample<NEST, NNZ, HWP, DEBUG, WIDE>(sl[j], x, pixelise, tod[j], g, a, cur.d0 + lane + 32 * j,
                                                             cur.s0 + k);
+#if !TB_DEFER
+                // fold this sample at once: no pending contribution is carried across iterations
+#pragma unroll
+                for (int j = 0; j < DPL; ++j) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, s_hits);
+#endif
             }
 
             if (nxt.item != cur.item) {
 #pragma unroll
                 for (int j = 0; j < DPL; ++j) {
-                    aggregate<NEST, NNZ, WIDE>(sl[j], a, g, s_hits);
+                    if (TB_DEFER) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, s_hits);
                     flush<NNZ, WIDE>(sl[j], a);
                 }
                 if (nxt.item < 0) break;
