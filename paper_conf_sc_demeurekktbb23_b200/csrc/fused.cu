@@ -254,6 +254,28 @@ struct Slot {
     bool ok;
 };
 
+// Per-CTA shared memory besides the warps' staging areas: the bit-spread table of the NEST
+// interleave (spread[b] = the 8 bits of b moved to the even bit positions) and the CTA's
+// hit-submap flags (MapGeom::shared_hits).
+struct CtaMem {
+    const uint16_t* spread;  // [256]
+    uint8_t* hits;           // [n_submap] when MapGeom::shared_hits
+};
+constexpr int kSpreadBytes = 512;
+
+// Pixel of a 32-bit run key with the bit interleave from the shared spread table: 2 (nside <=
+// 256) or 4 table loads instead of the ~16 instructions of interleave16 — this runs at every run
+// start, and with 32 detectors per warp some lane starts a run at most samples.
+template <bool NEST>
+__device__ __forceinline__ int key_to_pix_tab(int key, const HealpixGeom& g, const uint16_t* spread) {
+    if (!NEST) return key;
+    const int m = (int)g.nside - 1;
+    const uint32_t ix = (uint32_t)(key & m), iy = (uint32_t)((key >> g.order) & m);
+    uint32_t v = spread[ix & 255u] | ((uint32_t)spread[iy & 255u] << 1);
+    if (g.order > 8) v |= (spread[ix >> 8] | ((uint32_t)spread[iy >> 8] << 1)) << 16;
+    return (key & ~((1 << (2 * g.order)) - 1)) | (int)v;
+}
+
 // A run starts: mark its submap hit (as A2 does) and issue the global2local lookup now, so
 // the load latency is hidden behind the run's samples instead of stalling the flush.  The hit
 // flag is stored only when the lane's submap CHANGES: thousands of warps re-writing the same
@@ -261,10 +283,14 @@ struct Slot {
 // Sets sl.run_loc (-1: the submap has no storage) and sl.run_lp.
 template <bool NEST, bool WIDE>
 __device__ __forceinline__ void start_run(typename PixT<WIDE>::T key, const FusedArgs& a, const HealpixGeom& g,
-                                          Slot<typename PixT<WIDE>::T>& sl, uint8_t* s_hits) {
+                                          Slot<typename PixT<WIDE>::T>& sl, const CtaMem& cm) {
     using P = typename PixT<WIDE>::T;
     const MapGeom& mg = a.map;
-    const P pix = key_to_pix<NEST, WIDE>(key, g);
+    P pix;
+    if constexpr (WIDE)
+        pix = key;
+    else
+        pix = key_to_pix_tab<NEST>(key, g, cm.spread);
     P sm;
     if (mg.sm_shift >= 0) {
         sm = pix >> mg.sm_shift;
@@ -278,11 +304,11 @@ __device__ __forceinline__ void start_run(typename PixT<WIDE>::T key, const Fuse
         // the CTA's shared copy (idempotent store, no atomic; see the kernel end)
 #if TB_HITDEDUP
         if (sm != sl.last_sm) {
-            s_hits[sm] = 1;
+            cm.hits[sm] = 1;
             sl.last_sm = sm;
         }
 #else
-        s_hits[sm] = 1;
+        cm.hits[sm] = 1;
 #endif
     } else if (a.hit_submaps && sm != sl.last_sm) {
         a.hit_submaps[sm] = 1;
@@ -508,13 +534,13 @@ __device__ __forceinline__ void det_sample(Slot<typename PixT<WIDE>::T>& sl, con
 // run of an item flushes nothing: run_loc starts at -1.
 template <bool NEST, int NNZ, bool WIDE>
 __device__ __forceinline__ void aggregate(Slot<typename PixT<WIDE>::T>& sl, const FusedArgs& a,
-                                          const HealpixGeom& g, uint8_t* s_hits) {
+                                          const HealpixGeom& g, const CtaMem& cm) {
     if (sl.pend_key >= 0 && sl.pend_key != sl.run_key) {
 #ifndef TB_X_NOFLUSH
         flush<NNZ, WIDE>(sl, a);
 #endif
         sl.run_key = sl.pend_key;
-        start_run<NEST, WIDE>(sl.pend_key, a, g, sl, s_hits);
+        start_run<NEST, WIDE>(sl.pend_key, a, g, sl, cm);
         sl.r0 = sl.r1 = sl.r2 = 0.0;
     }
     sl.r0 += sl.p0;
@@ -586,13 +612,20 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
     // the alignment that matters for TMA and the swizzle is that of the shared-window offset)
     const unsigned pad1k = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
     TmaWarpSmem& tw = reinterpret_cast<TmaWarpSmem*>(smem_raw + pad1k)[wid];
-    // the CTA's hit-submap flags (MapGeom::shared_hits): after every warp's staging area
-    uint8_t* s_hits = smem_raw + (TMA ? 1024 + kWarps * sizeof(TmaWarpSmem) : kWarps * sizeof(WarpSmem<DPL>));
+    // the CTA's spread table and hit-submap flags: after every warp's staging area
+    unsigned char* cta_extra = smem_raw + (TMA ? 1024 + kWarps * sizeof(TmaWarpSmem) : kWarps * sizeof(WarpSmem<DPL>));
+    uint16_t* s_spread = reinterpret_cast<uint16_t*>(cta_extra);
+    uint8_t* s_hits = cta_extra + kSpreadBytes;
+    const CtaMem cm{s_spread, s_hits};
     const bool shared_hits = a.map.shared_hits;
-    if (shared_hits) {
-        for (int i = threadIdx.x; i < (int)a.map.n_submap; i += blockDim.x) s_hits[i] = 0;
-        __syncthreads();
+    for (int i = threadIdx.x; i < 256; i += blockDim.x) {
+        unsigned v = 0u;
+        for (int b = 0; b < 8; ++b) v |= ((i >> b) & 1u) << (2 * b);
+        s_spread[i] = (uint16_t)v;
     }
+    if (shared_hits)
+        for (int i = threadIdx.x; i < (int)a.map.n_submap; i += blockDim.x) s_hits[i] = 0;
+    __syncthreads();
     constexpr int kRows = 32 * DPL;
     const int64_t n_groups = (a.n_det + kRows - 1) / kRows;
     const int64_t n_items = n_chunks * n_groups;
@@ -822,7 +855,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
 #if TB_DEFER
                 // fold the previous sample while those shared-memory loads are in flight
 #pragma unroll
-                for (int j = 0; j < DPL; ++j) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, s_hits);
+                for (int j = 0; j < DPL; ++j) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, cm);
 #endif
 #pragma unroll
                 for (int j = 0; j < DPL; ++j)
@@ -831,14 +864,14 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
 #if !TB_DEFER
                 // fold this sample at once: no pending contribution is carried across iterations
 #pragma unroll
-                for (int j = 0; j < DPL; ++j) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, s_hits);
+                for (int j = 0; j < DPL; ++j) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, cm);
 #endif
             }
 
             if (nxt.item != cur.item) {
 #pragma unroll
                 for (int j = 0; j < DPL; ++j) {
-                    if (TB_DEFER) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, s_hits);
+                    if (TB_DEFER) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, cm);
                     flush<NNZ, WIDE>(sl[j], a);
                 }
                 if (nxt.item < 0) break;
@@ -954,7 +987,7 @@ cudaError_t launch_k(const WorkList& wl, const FusedArgs& a, const TmaMaps& tm, 
                      cudaStream_t st) {
     auto kern = pointing_to_map_kernel<NEST, NNZ, HWP, DEBUG, WIDE, DPL, TMA>;
     const size_t smem =
-        (TMA ? sizeof(TmaWarpSmem) * kWarps + 1024 : sizeof(WarpSmem<DPL>) * kWarps) + kSharedHitBytes;
+        (TMA ? sizeof(TmaWarpSmem) * kWarps + 1024 : sizeof(WarpSmem<DPL>) * kWarps) + kSpreadBytes + kSharedHitBytes;
     static int blocks_per_sm = 0;
     static std::once_flag once;
     std::call_once(once, [&] {
