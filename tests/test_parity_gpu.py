@@ -214,6 +214,42 @@ def test_fused_global2local_permuted():
     check_map(dw.zmap.cpu().numpy(), zo, absmap)
 
 
+def test_fused_compact_map_domain():
+    """f3 on the GPU: the hit submaps of a first pass define a compact (hit-submap-only)
+    global2local; the fused kernel accumulating into the compact map gives the oracle's dense
+    map on every hit submap (bench.py --reduce scatter runs exactly this)."""
+    from paper_conf_sc_demeurekktbb23_b200 import dist as tdist
+    w = synth.make_workload("c5", n_det=40, n_samp=40_000)
+    zo, absmap, ho, po, wo = _oracle_fused(w)
+    dw = DeviceWorkload.upload(w, DEV)
+    dw.pointing_to_map()
+    g2l, n_hit = tdist.compact_global2local(dw.hit_submaps)
+    assert 0 < n_hit < w.n_submap
+    own = tdist.MapOwnership.make(n_hit, 1)
+    zc = tdist.alloc_compact_map(own, w.n_pix_submap, w.nnz, DEV)
+    dw.global2local = g2l
+    dw.hit_submaps.zero_()
+    dw.pointing_to_map(zmap=zc)
+    torch.cuda.synchronize()
+    hit = np.nonzero(ho)[0]
+    np.testing.assert_array_equal(np.nonzero(dw.hit_submaps.cpu().numpy())[0], hit)
+    check_map(zc[:n_hit].cpu().numpy(), zo[hit], absmap[hit])
+    full = tdist.gather_map(zc[:own.per_rank], own, g2l, w.n_submap)
+    check_map(full.cpu().numpy(), zo, absmap)
+
+
+@pytest.mark.parametrize("dets", [(0, 0), (5, 6), (0, 33)])
+def test_fused_detector_counts(dets):
+    """No detector (a no-op), a single detector, one full warp group plus a one-detector group."""
+    w = synth.make_workload("c2", n_det=64, n_samp=30_000, det_range=dets)
+    zo, absmap, ho, po, wo = _oracle_fused(w)
+    dw = DeviceWorkload.upload(w, DEV)
+    dw.pointing_to_map()
+    torch.cuda.synchronize()
+    check_map(dw.zmap.cpu().numpy(), zo, absmap)
+    np.testing.assert_array_equal(dw.hit_submaps.cpu().numpy(), ho)
+
+
 # ----------------------------------------------------------------------------- unfused entries
 
 @pytest.fixture(scope="module")
