@@ -45,6 +45,7 @@ int cuda_fail(cudaError_t e, const char* where) {
 struct CacheEntry {
     int device;
     int chunk;
+    int64_t tail;  // the last `tail` in-interval samples are cut into chunks of kTailChunk
     std::vector<toast_interval_t> intervals;
     Chunk* d_chunks;
     int64_t n_chunks;
@@ -70,7 +71,11 @@ int validate_intervals(const toast_interval_t* iv, int64_t n, int64_t n_samp) {
 }
 
 // Returns the device work list for these intervals (creating it on first use).
-int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, WorkList* out, int chunk = kChunk) {
+// Chunk length of the work-list tail (see fused_worklist).
+constexpr int kTailChunk = 32;
+
+int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, WorkList* out, int chunk = kChunk,
+                 int64_t tail = 0) {
     int rc = validate_intervals(iv, n, n_samp);
     if (rc != TOAST_OK) return rc;
     int dev = 0;
@@ -78,19 +83,23 @@ int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, WorkList
     if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
     std::lock_guard<std::mutex> lk(g_cache_mu);
     for (auto& c : g_cache) {
-        if (c.device == dev && c.chunk == chunk && (int64_t)c.intervals.size() == n &&
+        if (c.device == dev && c.chunk == chunk && c.tail == tail && (int64_t)c.intervals.size() == n &&
             (n == 0 || std::memcmp(c.intervals.data(), iv, sizeof(toast_interval_t) * n) == 0)) {
             *out = WorkList{c.d_chunks, c.n_chunks, c.n_samples};
             return TOAST_OK;
         }
     }
     std::vector<Chunk> chunks;
+    int64_t all = 0;
+    for (int64_t i = 0; i < n; ++i) all += iv[i].last - iv[i].first + 1;
     int64_t total = 0;
     for (int64_t i = 0; i < n; ++i) {
-        for (int64_t f = iv[i].first; f <= iv[i].last; f += chunk) {
-            const int64_t cnt = std::min<int64_t>(chunk, iv[i].last - f + 1);
+        for (int64_t f = iv[i].first; f <= iv[i].last;) {
+            const int len = (total >= all - tail) ? kTailChunk : chunk;
+            const int64_t cnt = std::min<int64_t>(len, iv[i].last - f + 1);
             chunks.push_back(Chunk{f, (int32_t)cnt, (int32_t)i});
             total += cnt;
+            f += cnt;
         }
     }
     Chunk* d = nullptr;
@@ -114,21 +123,29 @@ int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, WorkList
         g_cache.erase(g_cache.begin());
     }
     g_cache.push_back(
-        CacheEntry{dev, chunk, std::vector<toast_interval_t>(iv, iv + n), d, (int64_t)chunks.size(), total});
+        CacheEntry{dev, chunk, tail, std::vector<toast_interval_t>(iv, iv + n), d, (int64_t)chunks.size(), total});
     *out = WorkList{d, (int64_t)chunks.size(), total};
     return TOAST_OK;
 }
 
 // Work list of the fused kernels: chunks of kFusedChunk samples, shorter when few detector groups
 // x few samples would leave the persistent grid idle (C1: 4 detectors, one group of 32 lanes),
-// so that there are at least ~4 items per resident warp.
+// so that there are at least ~4 items per resident warp.  Items are handed out in list order,
+// so the LAST items set the kernel's tail: a warp streams one 128-sample item for ~1/6 of the
+// C2 kernel time, and warps that draw no new item idle meanwhile.  The last ~2 items' worth of
+// samples per resident warp are therefore cut into kTailChunk-sample chunks.
 int fused_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, int64_t n_det, WorkList* out) {
     int rc = get_worklist(iv, n, n_samp, out, kFusedChunk);
     if (rc != TOAST_OK) return rc;
-    const int64_t groups = (n_det + 31) / 32, want = 4 * (int64_t)num_sms() * 16;
+    const int64_t groups = (n_det + 31) / 32, warps = (int64_t)num_sms() * 16, want = 4 * warps;
     int chunk = kFusedChunk;
     while (chunk > 16 && (out->n_samples / chunk) * groups < want) chunk /= 2;
-    return chunk == kFusedChunk ? TOAST_OK : get_worklist(iv, n, n_samp, out, chunk);
+#ifndef TB_NO_TAIL
+    const int64_t tail = chunk > kTailChunk ? std::min<int64_t>(out->n_samples / 4, 2 * warps * kTailChunk / groups) : 0;
+#else
+    const int64_t tail = 0;
+#endif
+    return (chunk == kFusedChunk && tail == 0) ? TOAST_OK : get_worklist(iv, n, n_samp, out, chunk, tail);
 }
 
 bool is_pow2(int64_t x) { return x > 0 && (x & (x - 1)) == 0; }
