@@ -130,13 +130,15 @@ def dist_env():
     return world, rank, local
 
 
-def algorithmic_bytes(w, det_samples: int) -> float:
-    """HBM bytes one step must move: TOD + det flags per det-sample,
-    boresight/HWP/shared flags per sample, one zeroing write + one write-back of the map."""
+def algorithmic_bytes(w, det_samples: int, touched_pixels: int) -> float:
+    """HBM bytes one launch of the fused kernel must move (SURVEY 8(d) B_alg, DESIGN.md
+    "Roofline"): TOD + det flags per det-sample, boresight/HWP/shared flags per sample, and one
+    read + one write-back of the map pixels the observation touches (the zeroing of the map is a
+    separate fill, outside the kernel)."""
     n_in = det_samples // w.n_det
     b = det_samples * (8 + (1 if w.det_flags is not None else 0))
     b += n_in * (32 + (8 if w.hwp is not None else 0) + (1 if w.shared_flags is not None else 0))
-    b += 2 * w.npix * w.nnz * 8
+    b += 2 * touched_pixels * w.nnz * 8
     return float(b)
 
 
@@ -326,7 +328,8 @@ def main():
     clk = clocks.get("sm_max_mhz") or 1965.0
     peak_tflops = SMS * DFMA_PER_SM_PER_CLK * 2 * clk * 1e6 / 1e12
     ach_tflops = F_ALG * det_samples / (kern_ms / 1e3) / 1e12
-    b_alg = algorithmic_bytes(w, det_samples)
+    touched = int(torch.count_nonzero(dw.zmap.reshape(-1, w.nnz).abs().sum(dim=1)))
+    b_alg = algorithmic_bytes(w, det_samples, touched)
     peaks = {}
     try:
         peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -351,6 +354,7 @@ def main():
                              "B200_PROFILING.md unit counts + nvidia-smi max clock)",
                 "hbm": {"achieved_gbs": b_alg / (kern_ms / 1e3) / 1e9, "peak_gbs": hbm_peak,
                         "frac": b_alg / (kern_ms / 1e3) / 1e9 / hbm_peak, "alg_bytes_per_launch": b_alg,
+                        "touched_pixels": touched,
                         "peak_note": "MEASURED_PEAKS.json hbm_gbs (measured)" if "hbm_gbs" in peaks
                         else "fallback 6650 GB/s"}}
 
