@@ -247,6 +247,7 @@ struct Slot {
     P run_lp;             // its pixel's index inside the submap
     int64_t run_loc;      // global2local of the run's submap, LOADED WHEN THE RUN STARTS
     P last_sm;            // last submap this lane marked in hit_submaps (generic path)
+    int64_t last_loc;     // SCAN: global2local of last_sm
     double r0, r1, r2;
     P pend_key;           // pending (not yet aggregated) det-sample
     double p0, p1, p2;
@@ -371,6 +372,7 @@ __device__ __forceinline__ void load_slot(Slot<P>& sl, const FusedArgs& a, int64
     sl.run_lp = 0;
     sl.run_loc = -1;
     sl.last_sm = -1;
+    sl.last_loc = -1;
     sl.r0 = sl.r1 = sl.r2 = 0.0;
     sl.pend_key = -1;
     sl.p0 = sl.p1 = sl.p2 = 0.0;
@@ -595,13 +597,19 @@ __device__ __forceinline__ void issue_block(RawBlock<DPL>& rb, const Blk& bk, co
     cp_async_commit();
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL, bool TMA>
+// SCAN = true: the scan direction, toast_pointing_to_tod: the same item / block
+// stream, staging and per-det-sample arithmetic, but each det-sample GATHERS its pixel's map
+// values (cached per lane across the run) and updates its TOD in the staged tile; the processed
+// columns of the tile are written back after each block (per-lane stores: a TMA store of the
+// whole box would overwrite samples of a neighbouring chunk that another warp owns).
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL, bool TMA, bool SCAN = false>
 __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_kernel(const Chunk* __restrict__ chunks,
                                                                          int64_t n_chunks, FusedArgs a,
                                                                          HealpixGeom g,
                                                                          unsigned long long* __restrict__ sched,
                                                                          const __grid_constant__ TmaMaps tm) {
     static_assert(!TMA || (DPL == 1 && kBlk == 16), "the TMA path stages 32 x 16 tiles");
+    static_assert(!SCAN || (DPL == 1 && !DEBUG), "the scan direction: one detector per lane, no debug outputs");
     using P = typename PixT<WIDE>::T;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int lane = threadIdx.x & 31;
@@ -631,12 +639,14 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
     const int64_t n_items = n_chunks * n_groups;
     const unsigned dmask = a.det_flag_mask;
     const unsigned smask = a.shared_flag_mask;
-    const bool have_dflags = a.det_flags != nullptr;
+    const bool have_dflags = !SCAN && a.det_flags != nullptr;  // scan_map ignores det flags (S12)
     const bool have_sflags = a.shared_flags != nullptr;
     // TMA: bytes landing per block (full boxes, out-of-range elements zero-filled)
     const unsigned tx_bytes = 32 * 16 * 8 + 16 * 32 + (have_dflags ? 32 * 16 : 0) +
                               ((HWP && NNZ == 3) ? 16 * 8 : 0) + (have_sflags ? 16 : 0);
     unsigned phase = 0u;  // TMA: bit b = parity of the next completion of mbar[b]
+    const double sgn_ds = (a.should_subtract ? -1.0 : 1.0) * a.data_scale;  // SCAN only
+    const double keep_old = a.should_zero ? 0.0 : 1.0;                       // SCAN only
     // swizzled byte offset of row `lane` in a TOD tile; sample k is at row_swz ^ (8 k)
     const unsigned row_swz = (unsigned)lane * 128u + (((unsigned)lane & 7u) << 4);
 
@@ -830,6 +840,67 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
             // TMA tile: the tile is 1 KB-aligned and row r starts at r * 128, so the swizzled address
             // of (lane, k) is (tile + row_swz) ^ (8 k): one LOP3 per sample.
             const unsigned tod_row = smem_u32(&tw.tod[p][0][0]) + row_swz;
+            // SCAN: the per-lane gather cache lives in the slot (run_key / run_loc: the cached
+            // pixel's key and storage; r0..r2 its map values; pend_key: the block sample whose TOD
+            // update waits for them, completed one sample later so the gather latency hides
+            // behind that sample)
+            auto store_tod = [&](int kk, double v) {
+                if constexpr (TMA)
+                    asm volatile("st.shared.f64 [%0], %1;" ::"r"(tod_row ^ ((unsigned)kk << 3)), "d"(v) : "memory");
+                else
+                    rb.tod[lane][kk] = v;
+            };
+            auto scan_finish = [&]() {
+                if constexpr (SCAN) {
+                    Slot<P>& s0 = sl[0];
+                    if (s0.pend_key >= 0) {
+                        double t = s0.r0 * a.cal;
+                        if (NNZ == 3) t += s0.etacal * (s0.r1 * s0.p1 + s0.r2 * s0.p2);
+                        store_tod((int)s0.pend_key, fma(sgn_ds, t, keep_old * s0.p0));
+                        s0.pend_key = -1;
+                    }
+                }
+            };
+            auto scan_sample = [&](int kk, const double* x, double tod) {
+                if constexpr (SCAN) {
+                    Slot<P>& s0 = sl[0];
+                    const StageA o = stage_a<NNZ, HWP, P>(s0, x);
+                    const P key = stage_b<NEST, NNZ, WIDE>(o, true, s0.ok, g);
+                    scan_finish();  // the previous sample's gathered values have arrived by now
+                    const MapGeom& mg = a.map;
+                    if (key >= 0 && key != s0.run_key) {
+                        P pix;
+                        if constexpr (WIDE)
+                            pix = key;
+                        else
+                            pix = key_to_pix_tab<NEST>(key, g, cm.spread);
+                        const int64_t smi = submap_of<P>(pix, mg);
+                        if (smi != (int64_t)s0.last_sm) {
+                            s0.last_loc = __ldg(&mg.global2local[smi]);
+                            s0.last_sm = (P)smi;
+                        }
+                        s0.run_key = key;
+                        s0.run_loc = s0.last_loc;
+                        if (s0.run_loc >= 0) {
+                            const int64_t lp = mg.sm_shift >= 0 ? (int64_t)(pix & (P)(mg.n_pix_submap - 1))
+                                                                : (int64_t)pix - smi * mg.n_pix_submap;
+                            const double* mp = a.mapdata + (s0.run_loc * mg.n_pix_submap + lp) * NNZ;
+                            s0.r0 = __ldg(mp);
+                            if (NNZ == 3) {
+                                s0.r1 = __ldg(mp + 1);
+                                s0.r2 = __ldg(mp + 2);
+                            }
+                        }
+                    }
+                    if (key >= 0 && s0.run_loc >= 0) {
+                        s0.pend_key = (P)kk;
+                        s0.p0 = tod;
+                        s0.p1 = o.cw * o.invr;
+                        s0.p2 = o.sw * o.invr;
+                    }
+                }
+            };
+
             int k = cur.k0;
             const int k_end = cur.k0 + cur.nb;
             unsigned bit = 1u << k;  // 1 << k
@@ -852,27 +923,54 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
                     else
                         tod[j] = rb.tod[lane + 32 * j][k];
                 }
+                if constexpr (SCAN) {
+                    scan_sample(k, x, tod[0]);
+                } else {
 #if TB_DEFER
-                // fold the previous sample while those shared-memory loads are in flight
+                    // fold the previous sample while those shared-memory loads are in flight
 #pragma unroll
-                for (int j = 0; j < DPL; ++j) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, cm);
+                    for (int j = 0; j < DPL; ++j) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, cm);
 #endif
 #pragma unroll
-                for (int j = 0; j < DPL; ++j)
-                    det_sample<NEST, NNZ, HWP, DEBUG, WIDE>(sl[j], x, pixelise, tod[j], g, a, cur.d0 + lane + 32 * j,
-                                                            cur.s0 + k);
+                    for (int j = 0; j < DPL; ++j)
+                        det_sample<NEST, NNZ, HWP, DEBUG, WIDE>(sl[j], x, pixelise, tod[j], g, a,
+                                                                cur.d0 + lane + 32 * j, cur.s0 + k);
 #if !TB_DEFER
-                // fold this sample at once: no pending contribution is carried across iterations
+                    // fold this sample at once: no pending contribution is carried across iterations
 #pragma unroll
-                for (int j = 0; j < DPL; ++j) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, cm);
+                    for (int j = 0; j < DPL; ++j) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, cm);
 #endif
+                }
+            }
+            if constexpr (SCAN) {
+                scan_finish();
+                __syncwarp();
+                // write back the processed columns of the tile (two rows per warp instruction,
+                // coalesced along samples); unprocessed samples in them keep the value read
+                const int scol = lane & 15, srow = lane >> 4;
+                if (scol >= cur.k0 && scol < cur.k0 + cur.nb) {
+                    double* dst = a.tod_out + (cur.d0 + srow) * a.n_samp + cur.s0 + scol;
+                    for (int r = srow; r < cur.nrows; r += 2, dst += 2 * a.n_samp) {
+                        double v;
+                        if constexpr (TMA)
+                            asm volatile("ld.shared.f64 %0, [%1];"
+                                         : "=d"(v)
+                                         : "r"(smem_u32(&tw.tod[p][0][0]) + (unsigned)r * 128u +
+                                               (((unsigned)scol << 3) ^ (((unsigned)r & 7u) << 4))));
+                        else
+                            v = rb.tod[r][scol];
+                        *dst = v;
+                    }
+                }
             }
 
             if (nxt.item != cur.item) {
 #pragma unroll
                 for (int j = 0; j < DPL; ++j) {
-                    if (TB_DEFER) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, cm);
-                    flush<NNZ, WIDE>(sl[j], a);
+                    if constexpr (!SCAN) {
+                        if (TB_DEFER) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, cm);
+                        flush<NNZ, WIDE>(sl[j], a);
+                    }
                 }
                 if (nxt.item < 0) break;
 #pragma unroll
@@ -982,10 +1080,10 @@ bool make_tma_maps(const FusedArgs& a, TmaMaps* tm) {
     return true;
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL, bool TMA>
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL, bool TMA, bool SCAN = false>
 cudaError_t launch_k(const WorkList& wl, const FusedArgs& a, const TmaMaps& tm, unsigned long long* sched,
                      cudaStream_t st) {
-    auto kern = pointing_to_map_kernel<NEST, NNZ, HWP, DEBUG, WIDE, DPL, TMA>;
+    auto kern = pointing_to_map_kernel<NEST, NNZ, HWP, DEBUG, WIDE, DPL, TMA, SCAN>;
     const size_t smem =
         (TMA ? sizeof(TmaWarpSmem) * kWarps + 1024 : sizeof(WarpSmem<DPL>) * kWarps) + kSpreadBytes + kSharedHitBytes;
     static int blocks_per_sm = 0;
@@ -1006,19 +1104,19 @@ cudaError_t launch_k(const WorkList& wl, const FusedArgs& a, const TmaMaps& tm, 
     return cudaGetLastError();
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL>
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL, bool SCAN = false>
 cudaError_t launch_t(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
     TmaMaps tm;
     if constexpr (kBlk == 16) {
         if (DPL == 1 && make_tma_maps(a, &tm)) {
             t_fused_path = "tma";
-            return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, 1, true>(wl, a, tm, sched, st);
+            return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, 1, true, SCAN>(wl, a, tm, sched, st);
         }
     } else {
         t_fused_path = "cp.async (8-sample blocks)";
     }
     std::memset(&tm, 0, sizeof(tm));
-    return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, DPL, false>(wl, a, tm, sched, st);
+    return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, DPL, false, SCAN>(wl, a, tm, sched, st);
 }
 
 template <bool NEST, int NNZ, bool HWP, bool DEBUG>
@@ -1044,224 +1142,15 @@ cudaError_t dispatch_hwp(const WorkList& wl, const FusedArgs& a, unsigned long l
 }
 
 // ============================================================================ scan direction
-// toast_pointing_to_tod: A1 -> A2 -> A3 -> A5 per det-sample in registers,
-// the map GATHERED into the timestream in place.  Same item / block stream and per-sample
-// state as pointing_to_map_kernel (lane = detector, cp.async double buffer); per lane the map
-// values of the current pixel are cached across the run (one gather per pixel change, the
-// submap's global2local cached across runs), and the TOD update of sample k is completed at
-// sample k+1 so the gather latency hides behind one sample of pointing work.  The block's
-// TOD tile is updated in shared memory and written back coalesced.
-template <bool NEST, int NNZ, bool HWP, bool WIDE>
-__global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_tod_kernel(const Chunk* __restrict__ chunks,
-                                                                         int64_t n_chunks, FusedArgs a,
-                                                                         HealpixGeom g,
-                                                                         unsigned long long* __restrict__ sched) {
-    using P = typename PixT<WIDE>::T;
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    const int lane = threadIdx.x & 31;
-    const int wid = threadIdx.x >> 5;
-    WarpSmem<1>& sm = reinterpret_cast<WarpSmem<1>*>(smem_raw)[wid];
-    const int64_t n_groups = (a.n_det + 31) / 32;
-    const int64_t n_items = n_chunks * n_groups;
-    const unsigned smask = a.shared_flag_mask;
-    const bool have_sflags = a.shared_flags != nullptr;
-    const MapGeom& mg = a.map;
-    const double ds = a.data_scale;
-    const double sgn = a.should_subtract ? -1.0 : 1.0;
-    const double keep = a.should_zero ? 0.0 : 1.0;
-
-    int64_t pend_item = -1, pend_first = 0;
-    int pend_count = 0;
-    auto prefetch_item = [&]() {
-        if (lane == 0) {
-            const unsigned long long it = atomicAdd(sched, 1ull);
-            pend_item = it < (unsigned long long)n_items ? (int64_t)it : -1;
-            if (pend_item >= 0) {
-                const Chunk ch = chunks[pend_item / n_groups];
-                pend_first = ch.first;
-                pend_count = ch.count;
-            }
-        }
-    };
-    auto take_item = [&]() -> Blk {
-        Blk bk;
-        bk.item = __shfl_sync(0xffffffffu, pend_item, 0);
-        const int64_t first = __shfl_sync(0xffffffffu, pend_first, 0);
-        const int count = __shfl_sync(0xffffffffu, pend_count, 0);
-        if (bk.item < 0) {
-            bk.d0 = bk.s0 = bk.s_end = 0;
-            bk.nb = bk.nrows = 0;
-            return bk;
-        }
-        const int64_t c = bk.item / n_groups;
-        bk.d0 = (bk.item - c * n_groups) * 32;
-        bk.nrows = (a.n_det - bk.d0) < 32 ? (int)(a.n_det - bk.d0) : 32;
-        bk.s0 = first;
-        bk.s_end = first + count;
-        bk.nb = count < kBlk ? count : kBlk;
-        return bk;
-    };
-
-    prefetch_item();
-    Blk cur = take_item();
-    if (cur.item < 0) return;
-    prefetch_item();
-    issue_block<1>(sm.buf[0], cur, a, false, HWP && NNZ == 3, lane);
-    Slot<P> sl;
-    load_slot<P>(sl, a, cur.d0 + lane, lane < cur.nrows, cur.d0);
-    int p = 0;
-    // per-lane gather cache: map values of the pixel of run key cur_key (loc < 0: no storage)
-    P cur_key = -1;
-    int64_t cur_loc = -1, last_sm = -1, last_loc = -1;
-    double m0 = 0.0, m1 = 0.0, m2 = 0.0;
-
-    while (true) {
-        Blk nxt;
-        if (cur.s0 + kBlk < cur.s_end) {
-            nxt = cur;
-            nxt.s0 = cur.s0 + kBlk;
-            nxt.nb = (nxt.s_end - nxt.s0) < kBlk ? (int)(nxt.s_end - nxt.s0) : kBlk;
-        } else {
-            nxt = take_item();
-            if (nxt.item >= 0) prefetch_item();
-        }
-        cp_async_wait_all();
-        __syncwarp();
-        if (nxt.item >= 0) issue_block<1>(sm.buf[p ^ 1], nxt, a, false, HWP && NNZ == 3, lane);
-
-        RawBlock<1>& rb = sm.buf[p];
-        bool pixelise_me = false;
-        if (lane < kBlk) {
-            double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 1.0;
-            double c4 = 1.0, s4 = 0.0;
-            if (lane < cur.nb) {
-                const int soff = have_sflags ? (int)(reinterpret_cast<uintptr_t>(a.shared_flags + cur.s0) & 3) : 0;
-                const bool flagged = have_sflags && (rb.sflg[soff + lane] & smask);
-                pixelise_me = !flagged;
-                if (!flagged) {
-                    q0 = rb.bore[lane][0]; q1 = rb.bore[lane][1]; q2 = rb.bore[lane][2]; q3 = rb.bore[lane][3];
-                }
-                if (HWP && NNZ == 3) small_sincos(4.0 * rb.hwp[lane], &s4, &c4);
-            }
-            SampleState x;
-            quat_to_matrix(q0, q1, q2, q3, x.v);
-            x.v[9] = c4;
-            x.v[10] = s4;
-            x.v[11] = 0.0;
-            sm.st[lane] = x;
-        }
-        const unsigned pmask = __ballot_sync(0xffffffffu, pixelise_me);
-        __syncwarp();
-
-        int pend_k = -1;  // sample whose TOD update waits for its gathered map values
-        double pend_tod = 0.0, pend_c2 = 0.0, pend_s2 = 0.0;
-        auto finish = [&]() {
-            if (pend_k >= 0) {
-                double t = m0 * a.cal;
-                if (NNZ == 3) t += sl.etacal * (m1 * pend_c2 + m2 * pend_s2);
-                rb.tod[lane][pend_k] = fma(sgn * ds, t, keep * pend_tod);
-                pend_k = -1;
-            }
-        };
-#pragma unroll 1
-        for (int k = 0; k < cur.nb; ++k) {
-            if (!((pmask >> k) & 1u)) continue;  // shared-flagged sample: no pixel, untouched (uniform)
-            double x[12];
-#pragma unroll
-            for (int i = 0; i < ((HWP && NNZ == 3) ? 12 : 10); i += 2) {
-                const double2 t2 = *reinterpret_cast<const double2*>(&sm.st[k].v[i]);
-                x[i] = t2.x;
-                x[i + 1] = t2.y;
-            }
-            const double tod = rb.tod[lane][k];
-            // the same per-det-sample arithmetic as pointing_to_map (incremental longitude,
-            // algebraic weights, run keys): cos 2psi' = cw / r, sin 2psi' = sw / r
-            const StageA o = stage_a<NNZ, HWP, P>(sl, x);
-            const P key = stage_b<NEST, NNZ, WIDE>(o, true, sl.ok, g);
-            const double c2 = o.cw * o.invr, s2 = o.sw * o.invr;
-            finish();  // the previous sample's gathered values have arrived by now
-            if (key >= 0 && key != cur_key) {
-                const P pix = key_to_pix<NEST, WIDE>(key, g);
-                const int64_t smi = submap_of<P>(pix, mg);
-                if (smi != last_sm) {
-                    last_loc = __ldg(&mg.global2local[smi]);
-                    last_sm = smi;
-                }
-                cur_key = key;  // the run key of the cached pixel
-                cur_loc = last_loc;
-                if (cur_loc >= 0) {
-                    const int64_t lp = mg.sm_shift >= 0 ? (int64_t)(pix & (P)(mg.n_pix_submap - 1))
-                                                        : (int64_t)pix - smi * mg.n_pix_submap;
-                    const double* mp = a.mapdata + (cur_loc * mg.n_pix_submap + lp) * NNZ;
-                    m0 = __ldg(mp);
-                    if (NNZ == 3) {
-                        m1 = __ldg(mp + 1);
-                        m2 = __ldg(mp + 2);
-                    }
-                }
-            }
-            if (key >= 0 && cur_loc >= 0) {
-                pend_k = k;
-                pend_tod = tod;
-                pend_c2 = c2;
-                pend_s2 = s2;
-            }
-        }
-        finish();
-        __syncwarp();
-        // write the updated tile back (samples without a pixel keep the value read)
-        {
-            const int scol = lane & (kBlk - 1);
-            const int srow = lane / kBlk;
-            if (scol < cur.nb) {
-                double* dst = a.tod_out + (cur.d0 + srow) * a.n_samp + cur.s0 + scol;
-                const int64_t step = kRowStep * a.n_samp;
-                for (int r = srow; r < cur.nrows; r += kRowStep, dst += step) *dst = rb.tod[r][scol];
-            }
-        }
-        if (nxt.item != cur.item) {
-            if (nxt.item < 0) break;
-            load_slot<P>(sl, a, nxt.d0 + lane, lane < nxt.nrows, nxt.d0);
-            cur_key = -1;
-            cur_loc = -1;
-        }
-        __syncwarp();
-        cur = nxt;
-        p ^= 1;
-    }
-    cp_async_wait_all();
-}
-
-template <bool NEST, int NNZ, bool HWP, bool WIDE>
-cudaError_t launch_scan_t(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
-    auto kern = pointing_to_tod_kernel<NEST, NNZ, HWP, WIDE>;
-    const size_t smem = sizeof(WarpSmem<1>) * kWarps;
-    static int blocks_per_sm = 0;
-    static std::once_flag once;
-    std::call_once(once, [&] {
-        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, kern, kWarps * 32, smem) != cudaSuccess ||
-            blocks_per_sm < 1)
-            blocks_per_sm = 1;
-    });
-    const int64_t n_items = wl.n_chunks * ((a.n_det + 31) / 32);
-    const int64_t want = (n_items + kWarps - 1) / kWarps;
-    const int64_t grid = std::min<int64_t>(want, (int64_t)num_sms() * blocks_per_sm);
-    if (grid <= 0) return cudaSuccess;
-    cudaError_t e = cudaMemsetAsync(sched, 0, sizeof(unsigned long long), st);
-    if (e != cudaSuccess) return e;
-    kern<<<(unsigned)grid, kWarps * 32, smem, st>>>(wl.chunks, wl.n_chunks, a, make_geom(a.nside), sched);
-    return cudaGetLastError();
-}
-
+// toast_pointing_to_tod: pointing_to_map_kernel<..., SCAN = true>.
 template <bool NEST, int NNZ>
 cudaError_t dispatch_scan(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
     const bool wide = a.nside > 8192;
     const bool hwp = a.hwp && NNZ == 3;
-    if (wide) return hwp ? launch_scan_t<NEST, NNZ, true, true>(wl, a, sched, st)
-                         : launch_scan_t<NEST, NNZ, false, true>(wl, a, sched, st);
-    return hwp ? launch_scan_t<NEST, NNZ, true, false>(wl, a, sched, st)
-               : launch_scan_t<NEST, NNZ, false, false>(wl, a, sched, st);
+    if (wide) return hwp ? launch_t<NEST, NNZ, true, false, true, 1, true>(wl, a, sched, st)
+                         : launch_t<NEST, NNZ, false, false, true, 1, true>(wl, a, sched, st);
+    return hwp ? launch_t<NEST, NNZ, true, false, false, 1, true>(wl, a, sched, st)
+               : launch_t<NEST, NNZ, false, false, false, 1, true>(wl, a, sched, st);
 }
 
 }  // namespace

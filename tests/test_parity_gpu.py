@@ -473,6 +473,8 @@ SCAN_CASES = {
     "c2_nnz1": dict(name="c2", n_det=12, n_samp=60_000, nnz=1),
     "c3_ring_flags": dict(name="c3", n_det=36, n_samp=30_000),
     "c5_nest_4096": dict(name="c5", n_det=20, n_samp=60_000),
+    # n_samp % 16 != 0: the cp.async staging path instead of the TMA path
+    "c2_cp_async_path": dict(name="c2", n_det=36, n_samp=60_003),
 }
 
 
