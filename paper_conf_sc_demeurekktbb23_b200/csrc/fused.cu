@@ -1,30 +1,29 @@
-// fused.cu — toast_pointing_to_map: A1 -> A2 -> A3 -> A4 per detector-sample in registers.
+// fused.cu — toast_pointing_to_map: A1 -> A2 -> A3 -> A4 per detector-sample in registers, and
+// (SCAN mode of the same kernel) toast_pointing_to_tod: A1 -> A2 -> A3 -> A5.
 //
-// Decomposition (B200-first, DESIGN.md "Fused kernel"):
+// Decomposition (B200-first, DESIGN.md §6.1):
 //   * A WARP owns a work item = (chunk of <= kFusedChunk consecutive in-interval samples,
-//     group of 32*DPL detectors); LANE = DETECTOR (each lane carries DPL detectors, d and
-//     d + 32).  Items are handed out dynamically (one atomic per item, fetched one item
-//     ahead) in chunk-major order, so the warps in flight cover a short time window of the
-//     focal plane and the sky footprint they scatter into stays L2-resident.
-//   * Each lane holds its detectors' frames in registers for the whole item:
+//     group of 32 detectors); LANE = DETECTOR.  Items are handed out dynamically (one atomic per
+//     item, fetched one item ahead) in chunk-major order, so the warps in flight cover a short
+//     time window of the focal plane and the sky footprint they scatter into stays L2-resident.
+//   * Each lane holds its detector's frame in registers for the whole item:
 //       u = R(f) z, v = R(f) x, w = R(f) y, det_scale*cal, det_scale*eta*cal.
-//   * An item is a STREAM OF BLOCKS of kBlk = 16 samples, software-pipelined through two
-//     warp-private shared-memory buffers: while block i is computed, cp.async already
-//     copies ALL raw inputs of block i+1 — the TOD tile [32*DPL detectors x 16 samples]
-//     (two rows per instruction, coalesced along samples), the det-flag rows, the 16
-//     boresight quaternions, HWP angles and shared flags — so no global-memory latency is
-//     on the critical path.  At the start of a block, lanes 0..15 turn the raw per-sample
-//     inputs into the per-sample state (boresight rotation matrix B — identity if
-//     shared-flagged, reading S2 — and cos/sin 4 chi); every lane then walks the 16
-//     samples reading that state as shared-memory BROADCASTS and its TOD / flags from the
-//     padded (bank-conflict-free) tile.  Boresight, HWP and shared flags are read from HBM
-//     once per 32*DPL detectors; every HBM stream is read coalesced.
-//   * Per det-sample: dir = B u, bx = (B v)_z, by = -(B w)_z (15 DP ops), the HEALPix
-//     pixel (quarter-turn arctangent with one reciprocal; 32-bit integer path up to nside
-//     8192), cos/sin 2psi algebraically, the HWP angle addition, det_scale * tod * w.
-//   * Map accumulation is RUN-LENGTH aggregated per lane along time: consecutive samples of
-//     one detector that fall in the same pixel are summed in registers and flushed with one
-//     fp64 `red` per Stokes component when the pixel changes (no shuffles at all).
+//   * An item is a STREAM OF BLOCKS of kBlk = 16 samples through two warp-private shared
+//     buffers: while block i is computed, lane 0's bulk tensor copies (TMA, mbarrier-completed;
+//     per-lane cp.async when the TMA constraints fail) stage block i+1 — the TOD tile [32 x 16]
+//     (128-byte swizzled), the det-flag rows, 16 boresight quaternions, HWP angles and shared
+//     flags.  Lanes 0..15 turn them into the per-sample state (boresight rotation matrix B —
+//     identity if shared-flagged, reading S2), lanes 16..31 into cos/sin 4 chi; every lane then
+//     walks the 16 samples reading that state as shared-memory broadcasts.  Boresight, HWP and
+//     shared flags are read from HBM once per 32 detectors.
+//   * Per det-sample: dir = B u, bx = (B v)_z, by = -(B w)_z, the longitude carried
+//     incrementally along the lane's samples (one reciprocal shared with the weights), the
+//     HEALPix run key, cos/sin 2psi algebraically, the HWP angle addition.
+//   * Map accumulation is RUN-LENGTH aggregated per lane along time: consecutive samples of one
+//     detector in the same pixel are summed in registers and flushed with one fp64 `red` per
+//     Stokes component when the pixel changes; hit-submap flags are gathered per CTA in shared
+//     memory.  SCAN mode gathers the map instead (cached per lane across the run) and updates
+//     the staged TOD tile, written back after each block.
 #include <cuda.h>  // CUtensorMap (the encoder is fetched through the runtime; no -lcuda)
 #include <cuda_runtime.h>
 #include <cudaTypedefs.h>
