@@ -1128,9 +1128,81 @@ cudaError_t dispatch_shape(const WorkList& wl, const FusedArgs& a, unsigned long
                : launch_t<NEST, NNZ, HWP, DEBUG, false, 1>(wl, a, sched, st);
 }
 
+// ============================================================================ few detectors
+// With fewer than kThinMaxDet detectors a 32-lane detector group leaves most lanes idle (C1: 4
+// detectors, 4 of 32 lanes).  Then THREAD = (chunk, detector): each thread builds its own
+// per-sample state from the boresight (consecutive threads share a chunk, so those loads are
+// L1 broadcasts) and runs the same per-det-sample arithmetic, run aggregation and flush as the
+// warp-per-item kernel (stage_a / stage_b / aggregate / flush), with the CTA's hit flags in
+// shared memory.
+constexpr int kThinMaxDet = 8;
+
+template <bool NEST, int NNZ, bool HWP, bool WIDE>
+__global__ void __launch_bounds__(256) pointing_to_map_thin_kernel(const Chunk* __restrict__ chunks, int64_t n_chunks,
+                                                                  FusedArgs a, HealpixGeom g) {
+    using P = typename PixT<WIDE>::T;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    uint16_t* s_spread = reinterpret_cast<uint16_t*>(smem_raw);
+    uint8_t* s_hits = smem_raw + kSpreadBytes;
+    const CtaMem cm{s_spread, s_hits};
+    for (int i = threadIdx.x; i < 256; i += blockDim.x) {
+        unsigned v = 0u;
+        for (int b = 0; b < 8; ++b) v |= ((i >> b) & 1u) << (2 * b);
+        s_spread[i] = (uint16_t)v;
+    }
+    if (a.map.shared_hits)
+        for (int i = threadIdx.x; i < (int)a.map.n_submap; i += blockDim.x) s_hits[i] = 0;
+    __syncthreads();
+    const int64_t n_items = n_chunks * a.n_det;
+    for (int64_t it = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; it < n_items;
+         it += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t c = it / a.n_det, d = it - c * a.n_det;
+        const Chunk ch = chunks[c];
+        Slot<P> sl;
+        load_slot<P>(sl, a, d, true, d);
+        for (int64_t s = ch.first; s < ch.first + ch.count; ++s) {
+            if (a.shared_flags && (__ldg(&a.shared_flags[s]) & a.shared_flag_mask)) continue;  // no pixel (S2)
+            const double2 q01 = __ldg(reinterpret_cast<const double2*>(a.boresight + 4 * s));
+            const double2 q23 = __ldg(reinterpret_cast<const double2*>(a.boresight + 4 * s) + 1);
+            double x[12];
+            quat_to_matrix(q01.x, q01.y, q23.x, q23.y, x);
+            if (HWP && NNZ == 3) small_sincos(4.0 * __ldg(&a.hwp[s]), &x[10], &x[9]);
+            double tod = __ldg(&a.det_data[d * a.n_samp + s]);
+            if (a.det_flags && (__ldg(&a.det_flags[d * a.n_samp + s]) & a.det_flag_mask)) tod = 0.0;
+            aggregate<NEST, NNZ, WIDE>(sl, a, g, cm);
+            det_sample<NEST, NNZ, HWP, false, WIDE>(sl, x, true, tod, g, a, d, s);
+        }
+        aggregate<NEST, NNZ, WIDE>(sl, a, g, cm);
+        flush<NNZ, WIDE>(sl, a);
+    }
+    if (a.map.shared_hits) {
+        __syncthreads();
+        for (int i = threadIdx.x; i < (int)a.map.n_submap; i += blockDim.x)
+            if (s_hits[i]) a.hit_submaps[i] = 1;
+    }
+}
+
+template <bool NEST, int NNZ, bool HWP>
+cudaError_t launch_thin(const WorkList& wl, const FusedArgs& a, cudaStream_t st) {
+    const size_t smem = kSpreadBytes + kSharedHitBytes;
+    const int64_t items = wl.n_chunks * a.n_det;
+    const int64_t grid = std::min<int64_t>((items + 255) / 256, (int64_t)num_sms() * 8);
+    t_fused_path = "thin (thread per chunk x detector, few detectors)";
+    if (a.nside > 8192)
+        pointing_to_map_thin_kernel<NEST, NNZ, HWP, true><<<(unsigned)grid, 256, smem, st>>>(wl.chunks, wl.n_chunks, a,
+                                                                                              make_geom(a.nside));
+    else
+        pointing_to_map_thin_kernel<NEST, NNZ, HWP, false><<<(unsigned)grid, 256, smem, st>>>(wl.chunks, wl.n_chunks, a,
+                                                                                               make_geom(a.nside));
+    return cudaGetLastError();
+}
+
 template <bool NEST, int NNZ, bool HWP>
 cudaError_t dispatch_debug(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
     if (a.pixels_out || a.weights_out) return dispatch_shape<NEST, NNZ, HWP, true>(wl, a, sched, st);
+#ifndef TB_NO_THIN
+    if (a.n_det < kThinMaxDet) return launch_thin<NEST, NNZ, HWP>(wl, a, st);
+#endif
     return dispatch_shape<NEST, NNZ, HWP, false>(wl, a, sched, st);
 }
 

@@ -37,6 +37,13 @@ def _need_gpu():
     binding.load()
 
 
+def _assert_bench_path(w):
+    """The staging path bench.py times on this workload: TMA, or the thread-per-(chunk, detector)
+    kernel below 8 detectors (C1)."""
+    path = binding.last_fused_path()
+    assert path == "tma" or (w.n_det < 8 and path.startswith("thin")), path
+
+
 def _valid_mask_counts(w):
     """Per detector: number of in-interval samples that are neither shared- nor det-flagged."""
     inside = np.zeros(w.n_samp, bool)
@@ -72,7 +79,7 @@ def test_full_size_hit_count_property(name):
     w.cal = 1.0
     dw.pointing_to_map()
     torch.cuda.synchronize()
-    assert binding.last_fused_path() == "tma", binding.last_fused_path()
+    _assert_bench_path(w)
     del ones
     z = dw.zmap
     n_valid = int(_valid_mask_counts(w).sum())
@@ -150,7 +157,7 @@ def test_full_size_sparse_probes(name):
     dw = DeviceWorkload.upload(w, DEV, det_data=tod)
     dw.pointing_to_map()
     torch.cuda.synchronize()
-    assert binding.last_fused_path() == "tma", binding.last_fused_path()
+    _assert_bench_path(w)
     del tod
 
     keys = sorted(expect)
@@ -181,7 +188,7 @@ def test_full_size_whole_map(name):
     dw = DeviceWorkload.upload(w, DEV)
     dw.pointing_to_map()  # production instantiation, as bench.py times it
     torch.cuda.synchronize()
-    assert binding.last_fused_path() == "tma", binding.last_fused_path()
+    _assert_bench_path(w)
     zg = dw.zmap.cpu().numpy()
     hg = dw.hit_submaps.cpu().numpy()
 
