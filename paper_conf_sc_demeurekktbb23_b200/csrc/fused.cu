@@ -67,6 +67,9 @@ constexpr int kKUnroll = TB_KUNROLL;  // unroll of the per-sample loop
 #ifndef TB_TTOFF
 #define TB_TTOFF 1  // 32-bit keys: longitude carried as tt + 1 without wrapping (see stage_a)
 #endif
+#ifndef TB_INCR_BF
+#define TB_INCR_BF 1  // branch-free incremental-longitude series (see stage_a; measured -0.5..1 % C2)
+#endif
 #ifndef TB_DEFER
 #define TB_DEFER 1  // a det-sample's contribution is folded into its run one sample later
 #endif
@@ -424,6 +427,26 @@ __device__ __forceinline__ StageA stage_a(Slot<P>& sl, const double* x) {
         // |cross| < kIncrMax dot  <=>  dot > 0 and |t| < kIncrMax (t = cross / dot); false at
         // dot = 0 (no previous sample) and for steps beyond a quarter turn; one DFMA + DSETP,
         // resolved before the reciprocal's result is needed
+#if TB_INCR_BF
+        // branch-free common path: the series is evaluated for every sample (NaN at dot = 0, no
+        // traps on the GPU) and only the rare full-arctangent path is a branch, so the scheduler
+        // can interleave the series with the surrounding straight-line code
+        {
+            const double t = cross * (r * inv);
+            o.invr = dot * inv;
+            const double s2 = t * t;
+            double q = fma(kIncrQ[3], s2, kIncrQ[2]);
+            q = fma(q, s2, kIncrQ[1]);
+            q = fma(q, s2, kIncrQ[0]);
+            double tt = fma(t, q, sl.ptt);
+            if constexpr (!TTOFF) {
+                if (__double2hiint(tt) < 0) tt += 4.0;
+                if (__double2hiint(tt) >= 0x40100000) tt -= 4.0;
+            }
+            o.tt = tt;
+        }
+        if (!(fma(TB_INCR_MAX, dot, -fabs(cross)) > 0.0)) {
+#else
         if (fma(TB_INCR_MAX, dot, -fabs(cross)) > 0.0) {
             const double t = cross * (r * inv);
             o.invr = dot * inv;
@@ -438,6 +461,7 @@ __device__ __forceinline__ StageA stage_a(Slot<P>& sl, const double* x) {
             }
             o.tt = tt;
         } else {
+#endif
             // TTOFF: the chain is carried as tt + 1 WITHOUT wrapping: it restarts here from a
             // value in [1, 5) and drifts by at most 127 steps of (2/pi) atan(0.01) = 0.0064
             // within an item, so it stays in (0.18, 5.82); loc2key32<NEST, true> folds it back
