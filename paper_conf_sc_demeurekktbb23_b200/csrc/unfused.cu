@@ -169,6 +169,11 @@ __global__ void __launch_bounds__(kChunk) stokes_weights_kernel(
 
 // ----------------------------------------------------------------------------- A4
 
+#ifndef TB_A4_DT
+#define TB_A4_DT 1
+#endif
+constexpr int kA4DT = TB_A4_DT;
+
 template <int NNZ, bool IDX>
 __global__ void __launch_bounds__(kChunk) build_noise_weighted_kernel(
     const Chunk* __restrict__ chunks, int64_t n_chunks, MapGeom mg, double* __restrict__ zmap,
@@ -185,28 +190,40 @@ __global__ void __launch_bounds__(kChunk) build_noise_weighted_kernel(
         const bool in = (int)threadIdx.x < ch.count;
         const int64_t s = ch.first + threadIdx.x;
         const bool sflag = in && shared_flags && (__ldg(&shared_flags[s]) & shared_flag_mask);
-        // one detector per CTA row (batching detectors here raised registers and was slower)
-        for (int64_t d = blockIdx.y; d < n_det; d += gridDim.y) {
-            int64_t key = -1 - lane;
-            double v0 = 0.0, v1 = 0.0, v2 = 0.0;
-            if (in && !sflag) {
-                // all loads unconditional (no load waits on another before it is issued)
-                const int64_t pix = __ldg(&pixels[row_of<IDX>(pixel_index, d) * n_samp + s]);
-                const bool dflag =
-                    det_flags && (__ldg(&det_flags[row_of<IDX>(flag_index, d) * n_samp + s]) & det_flag_mask);
-                const double scaled = __ldg(&det_scale[d]) * __ldg(&det_data[row_of<IDX>(data_index, d) * n_samp + s]);
-                const double* w = weights + (row_of<IDX>(weight_index, d) * n_samp + s) * NNZ;
-                const double w0 = __ldg(&w[0]);
-                const double w1 = NNZ == 3 ? __ldg(&w[1]) : 0.0;
-                const double w2 = NNZ == 3 ? __ldg(&w[2]) : 0.0;
-                if (pix >= 0 && !dflag) {
-                    key = pix;
-                    v0 = scaled * w0;
-                    v1 = scaled * w1;
-                    v2 = scaled * w2;
+        // kA4DT detector rows per CTA row: every row's loads are issued before the first row's
+        // segmented scan, so each thread keeps kA4DT x 6 loads in flight
+        for (int64_t d0 = (int64_t)blockIdx.y * kA4DT; d0 < n_det; d0 += (int64_t)gridDim.y * kA4DT) {
+            int64_t key[kA4DT];
+            double v0[kA4DT], v1[kA4DT], v2[kA4DT];
+#pragma unroll
+            for (int j = 0; j < kA4DT; ++j) {
+                const int64_t d = d0 + j;
+                key[j] = -1 - lane;
+                v0[j] = v1[j] = v2[j] = 0.0;
+                if (in && !sflag && d < n_det) {
+                    // all loads unconditional (no load waits on another before it is issued)
+                    const int64_t pix = __ldg(&pixels[row_of<IDX>(pixel_index, d) * n_samp + s]);
+                    const bool dflag =
+                        det_flags && (__ldg(&det_flags[row_of<IDX>(flag_index, d) * n_samp + s]) & det_flag_mask);
+                    const double scaled =
+                        __ldg(&det_scale[d]) * __ldg(&det_data[row_of<IDX>(data_index, d) * n_samp + s]);
+                    const double* w = weights + (row_of<IDX>(weight_index, d) * n_samp + s) * NNZ;
+                    const double w0 = __ldg(&w[0]);
+                    const double w1 = NNZ == 3 ? __ldg(&w[1]) : 0.0;
+                    const double w2 = NNZ == 3 ? __ldg(&w[2]) : 0.0;
+                    if (pix >= 0 && !dflag) {
+                        key[j] = pix;
+                        v0[j] = scaled * w0;
+                        v1[j] = scaled * w1;
+                        v2[j] = scaled * w2;
+                    }
                 }
             }
-            warp_accumulate<NNZ>(key, v0, v1, v2, mg, zmap, nullptr);
+#pragma unroll
+            for (int j = 0; j < kA4DT; ++j) {
+                if (d0 + j >= n_det) break;
+                warp_accumulate<NNZ>(key[j], v0[j], v1[j], v2[j], mg, zmap, nullptr);
+            }
         }
     }
 }
@@ -308,11 +325,11 @@ cudaError_t launch_build_noise_weighted(const WorkList& wl, const MapGeom& mg, d
                                         uint8_t shared_flag_mask, int64_t n_det, int64_t n_samp, cudaStream_t st) {
     if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
     if (nnz == 3)
-        (pixel_index || weight_index || data_index || flag_index ? build_noise_weighted_kernel<3, true> : build_noise_weighted_kernel<3, false>)<<<grid_for(wl, n_det, 1), kChunk, 0, st>>>(
+        (pixel_index || weight_index || data_index || flag_index ? build_noise_weighted_kernel<3, true> : build_noise_weighted_kernel<3, false>)<<<grid_for(wl, n_det, kA4DT), kChunk, 0, st>>>(
             wl.chunks, wl.n_chunks, mg, zmap, pixel_index, pixels, weight_index, weights, data_index, det_data,
             flag_index, det_flags, det_flag_mask, det_scale, shared_flags, shared_flag_mask, n_det, n_samp);
     else
-        (pixel_index || weight_index || data_index || flag_index ? build_noise_weighted_kernel<1, true> : build_noise_weighted_kernel<1, false>)<<<grid_for(wl, n_det, 1), kChunk, 0, st>>>(
+        (pixel_index || weight_index || data_index || flag_index ? build_noise_weighted_kernel<1, true> : build_noise_weighted_kernel<1, false>)<<<grid_for(wl, n_det, kA4DT), kChunk, 0, st>>>(
             wl.chunks, wl.n_chunks, mg, zmap, pixel_index, pixels, weight_index, weights, data_index, det_data,
             flag_index, det_flags, det_flag_mask, det_scale, shared_flags, shared_flag_mask, n_det, n_samp);
     return cudaGetLastError();
