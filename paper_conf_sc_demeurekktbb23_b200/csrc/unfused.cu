@@ -44,12 +44,30 @@ dim3 grid_for(const WorkList& wl, int64_t n_det, int dt = kDT) {
     return dim3(gx, gy, 1);
 }
 
+// Resident 256-thread CTAs per SM each kernel's register allocation is bounded for (latency-bound
+// streaming kernels: more resident warps, more loads in flight).
+#ifndef TB_A1_MINB
+#define TB_A1_MINB 1
+#endif
+#ifndef TB_A2_MINB
+#define TB_A2_MINB 4  // measured on B200 (C2/C3): -26 % vs unbounded (80 registers -> 64)
+#endif
+#ifndef TB_A3_MINB
+#define TB_A3_MINB 1  // bounded variants spill (272+ bytes of stack) and run 50 % slower
+#endif
+#ifndef TB_A4_MINB
+#define TB_A4_MINB 8  // measured: -21 % (46 registers -> 32, 5 -> 8 resident CTAs)
+#endif
+#ifndef TB_A5_MINB
+#define TB_A5_MINB 8  // measured: -28 % (37 -> 32 registers)
+#endif
+
 #define FOR_DET_TILES(d0) for (int64_t d0 = (int64_t)blockIdx.y * kDT; d0 < n_det; d0 += (int64_t)gridDim.y * kDT)
 
 // ----------------------------------------------------------------------------- A1
 
 template <bool IDX>
-__global__ void __launch_bounds__(kChunk) pointing_detector_kernel(
+__global__ void __launch_bounds__(kChunk, TB_A1_MINB) pointing_detector_kernel(
     const Chunk* __restrict__ chunks, int64_t n_chunks, const double* __restrict__ fp_quats,
     const double* __restrict__ boresight, const int32_t* __restrict__ quat_index, double* __restrict__ quats,
     const uint8_t* __restrict__ shared_flags, uint8_t shared_flag_mask, int64_t n_det, int64_t n_samp) {
@@ -82,7 +100,7 @@ __global__ void __launch_bounds__(kChunk) pointing_detector_kernel(
 // ----------------------------------------------------------------------------- A2
 
 template <bool NEST, bool IDX>
-__global__ void __launch_bounds__(kChunk) pixels_healpix_kernel(
+__global__ void __launch_bounds__(kChunk, TB_A2_MINB) pixels_healpix_kernel(
     const Chunk* __restrict__ chunks, int64_t n_chunks, const int32_t* __restrict__ quat_index,
     const double* __restrict__ quats, const uint8_t* __restrict__ shared_flags, uint8_t shared_flag_mask,
     const int32_t* __restrict__ pixel_index, int64_t* __restrict__ pixels, uint8_t* __restrict__ hit_submaps,
@@ -127,7 +145,7 @@ __global__ void __launch_bounds__(kChunk) pixels_healpix_kernel(
 // ----------------------------------------------------------------------------- A3
 
 template <bool HWP, bool IDX>
-__global__ void __launch_bounds__(kChunk) stokes_weights_kernel(
+__global__ void __launch_bounds__(kChunk, TB_A3_MINB) stokes_weights_kernel(
     const Chunk* __restrict__ chunks, int64_t n_chunks, const int32_t* __restrict__ quat_index,
     const double* __restrict__ quats, const int32_t* __restrict__ weight_index, double* __restrict__ weights,
     const double* __restrict__ hwp, const double* __restrict__ epsilon, double cal, int64_t n_det, int64_t n_samp) {
@@ -170,12 +188,12 @@ __global__ void __launch_bounds__(kChunk) stokes_weights_kernel(
 // ----------------------------------------------------------------------------- A4
 
 #ifndef TB_A4_DT
-#define TB_A4_DT 1
+#define TB_A4_DT 1  // measured on B200 (C2): 2 rows per CTA row -4 %, 4 rows -40 % (registers)
 #endif
 constexpr int kA4DT = TB_A4_DT;
 
 template <int NNZ, bool IDX>
-__global__ void __launch_bounds__(kChunk) build_noise_weighted_kernel(
+__global__ void __launch_bounds__(kChunk, TB_A4_MINB) build_noise_weighted_kernel(
     const Chunk* __restrict__ chunks, int64_t n_chunks, MapGeom mg, double* __restrict__ zmap,
     const int32_t* __restrict__ pixel_index, const int64_t* __restrict__ pixels,
     const int32_t* __restrict__ weight_index, const double* __restrict__ weights,
@@ -231,7 +249,7 @@ __global__ void __launch_bounds__(kChunk) build_noise_weighted_kernel(
 // ----------------------------------------------------------------------------- A5
 
 template <int NNZ, bool IDX>
-__global__ void __launch_bounds__(kChunk) scan_map_kernel(
+__global__ void __launch_bounds__(kChunk, TB_A5_MINB) scan_map_kernel(
     const Chunk* __restrict__ chunks, int64_t n_chunks, MapGeom mg, const double* __restrict__ mapdata,
     const int32_t* __restrict__ data_index, double* __restrict__ det_data, const int32_t* __restrict__ pixel_index,
     const int64_t* __restrict__ pixels, const int32_t* __restrict__ weight_index, const double* __restrict__ weights,
