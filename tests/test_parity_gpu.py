@@ -238,9 +238,10 @@ def test_fused_compact_map_domain():
     check_map(full.cpu().numpy(), zo, absmap)
 
 
-@pytest.mark.parametrize("dets", [(0, 0), (5, 6), (0, 33)])
+@pytest.mark.parametrize("dets", [(0, 0), (5, 6), (0, 7), (0, 8), (0, 33)])
 def test_fused_detector_counts(dets):
-    """No detector (a no-op), a single detector, one full warp group plus a one-detector group."""
+    """No detector (a no-op), one and seven detectors (the thread-per-(chunk, detector) path), eight
+    (the warp path with 24 idle lanes), one full warp group plus a one-detector group."""
     w = synth.make_workload("c2", n_det=64, n_samp=30_000, det_range=dets)
     zo, absmap, ho, po, wo = _oracle_fused(w)
     dw = DeviceWorkload.upload(w, DEV)
