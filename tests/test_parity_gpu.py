@@ -183,6 +183,35 @@ def test_fused_extreme_nside(nside, nest):
     check_map(dw.zmap.cpu().numpy(), zo_r, abs_r)
 
 
+@pytest.mark.parametrize("name,n_det", [("c1", 4), ("c2", 40)])  # thread path and warp path
+def test_fused_production_wide_and_many_submaps(name, n_det):
+    """Production calls (no debug outputs) on the paths the tests above reach only with debug
+    outputs: 64-bit keys (nside 2^16, hit submaps only) and more than 8192 submaps (the hit flags
+    then go straight to global memory instead of the CTA's shared copy)."""
+    # nside 2^16: no storage, the hit submaps against the oracle's A2
+    w = synth.make_workload(name, n_det=n_det, n_samp=20_000, nside=1 << 16, nest=True)
+    quats = oracle.pointing_detector(w.fp_quats, w.boresight, w.intervals, w.shared_flags, w.shared_flag_mask)
+    _, hits = oracle.pixels_healpix(quats, w.intervals, w.nside, w.nest, w.n_pix_submap, w.shared_flags,
+                                    w.shared_flag_mask)
+    dw = DeviceWorkload.upload(w, DEV, alloc_map=False)
+    dw.global2local = torch.full((w.n_submap,), -1, dtype=torch.int64, device=DEV)
+    dw.pointing_to_map()
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(dw.hit_submaps.cpu().numpy(), hits)
+    # nside 64 with 4-pixel submaps: 12288 submaps
+    w = synth.make_workload(name, n_det=n_det, n_samp=20_000, nside=64)
+    w.n_pix_submap = 4
+    zo, absmap, ho, po, wo = _oracle_fused(w)
+    dw = DeviceWorkload.upload(w, DEV, alloc_map=False)
+    dw.zmap = torch.zeros(zo.shape, dtype=torch.float64, device=DEV)
+    dw.hit_submaps = torch.zeros(w.n_submap, dtype=torch.uint8, device=DEV)
+    assert w.n_submap > 8192
+    dw.pointing_to_map()
+    torch.cuda.synchronize()
+    check_map(dw.zmap.cpu().numpy(), zo, absmap)
+    np.testing.assert_array_equal(dw.hit_submaps.cpu().numpy(), ho)
+
+
 @pytest.mark.parametrize("n_samp", [5000, 5008])  # cp.async path (n_samp % 16 != 0) and TMA path
 def test_fused_edge_intervals(n_samp):
     """Empty interval list, single-sample intervals, chunk-boundary lengths (255/256/257),
