@@ -74,7 +74,7 @@ constexpr int kKUnroll = TB_KUNROLL;  // unroll of the per-sample loop
 #define TB_DEFER 1  // a det-sample's contribution is folded into its run one sample later
 #endif
 #ifndef TB_HITDEDUP
-#define TB_HITDEDUP 1  // shared hit flags: store only when the lane's submap changes
+#define TB_HITDEDUP 0  // shared hit flags: compare with the lane's last submap first (measured: +1 % C2, +2 % C3)
 #endif
 constexpr int kPad = kBlk + 1;
 
