@@ -12,7 +12,11 @@ namespace toastb200 {
 constexpr int kChunk = 256;
 // Samples per work chunk of the fused kernel (a warp item = one such chunk x 32 or 64
 // detectors; small enough that the dynamic schedule balances to a few percent).
-constexpr int kFusedChunk = 128;
+#ifndef TB_FUSED_CHUNK
+#define TB_FUSED_CHUNK 128  // <= 128: the incremental longitude's unwrapped range (fused.cu stage_a)
+#endif
+constexpr int kFusedChunk = TB_FUSED_CHUNK;
+static_assert(kFusedChunk <= 128, "the tt + 1 chain must stay inside (0.18, 5.82)");
 
 // One chunk of <= kChunk consecutive in-interval samples (never crosses an interval).
 struct Chunk {
