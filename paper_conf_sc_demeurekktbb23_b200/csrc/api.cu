@@ -144,7 +144,10 @@ int fused_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, int64_
     int rc = get_worklist(iv, n, n_samp, out, kFusedChunk);
     if (rc != TOAST_OK) return rc;
     const int64_t groups = (n_det + 31) / 32, warps = (int64_t)num_sms() * 16, want = 4 * warps;
-    int chunk = kFusedChunk;
+    // large focal planes (>= 64 detector groups: C4, C5) take 64-sample chunks: the warps in flight
+    // then span half the time window, so the map lines they scatter into are reused more in L2
+    // (measured: C5 -1.6 %; no effect below 64 groups, where the tail dominates)
+    int chunk = groups >= 64 ? kFusedChunk / 2 : kFusedChunk;
     while (chunk > 16 && (out->n_samples / chunk) * groups < want) chunk /= 2;
 #ifndef TB_NO_TAIL
     const int64_t tail = chunk > kTailChunk ? std::min<int64_t>(out->n_samples / 4, TB_TAIL_ITEMS * warps * kTailChunk / groups) : 0;
