@@ -66,6 +66,8 @@ def _declare(L):
     L.oracle_near_boundary.argtypes = [I64, INT, P, D]
     L.oracle_near_boundary.restype = INT
     L.oracle_stokes_iqu.argtypes = [P, D, D, D, P]
+    L.oracle_stokes_iqu_ex.argtypes = [P, INT, D, D, INT, D, D, P]
+    L.oracle_stokes_weights_iqu_ex.argtypes = [P, P, P, P, P, P, P, INT, D, P, I64, I64, I64]
     L.oracle_pointing_detector.argtypes = [P, P, P, P, P, I64, P, U8, I64, I64]
     L.oracle_pixels_healpix.argtypes = [P, P, P, U8, P, P, P, I64, P, I64, I64, INT, I64, I64]
     L.oracle_stokes_weights_iqu.argtypes = [P, P, P, P, P, P, D, P, I64, I64, I64]
@@ -74,12 +76,17 @@ def _declare(L):
     L.oracle_scan_map.argtypes = [P, I64, P, I64, P, P, P, P, P, P, P, I64, D, INT, INT, I64, I64, P]
     L.oracle_pointing_to_map.argtypes = [P, P, P, P, D, P, P, P, U8, P, U8, P, I64, I64, INT, I64, P, I64, P, P,
                                          P, P, I64, I64, P]
+    L.oracle_pointing_to_map_ex.argtypes = [P, P, P, P, D, P, P, P, U8, P, U8, P, I64, I64, INT, I64, P, I64, P,
+                                            P, P, P, I64, I64, P, P, INT]
     L.oracle_pointing_to_map_omp.argtypes = [P, P, P, P, D, P, P, P, U8, P, U8, P, I64, I64, INT, I64, P, I64,
                                              P, I64, I64, INT]
     L.oracle_pointing_to_map_omp.restype = INT
     L.oracle_det_sample_probe.argtypes = [P, P, D, D, D, INT, I64, INT, P, P, P]
+    L.oracle_det_sample_probe_ex.argtypes = [P, P, INT, D, D, INT, D, D, INT, I64, INT, P, P, P]
     L.oracle_pointing_to_tod.argtypes = [P, P, P, P, D, P, U8, P, I64, I64, INT, I64, P, I64, P, D, INT, INT, P, I64,
                                          I64, P]
+    L.oracle_pointing_to_tod_ex.argtypes = [P, P, P, P, D, P, U8, P, I64, I64, INT, I64, P, I64, P, D, INT, INT, P,
+                                            I64, I64, P, P, INT]
 
 
 def _p(a):
@@ -134,19 +141,24 @@ def near_boundary(nside: int, nest: bool, v, delta: float = 1.1e-12) -> bool:
     return bool(lib().oracle_near_boundary(nside, int(nest), _p(v), delta))
 
 
-def stokes_iqu(q, hwp_angle: float, epsilon: float, cal: float):
+def stokes_iqu(q, hwp_angle, epsilon: float, cal: float, gamma: float = 0.0, iau: bool = False):
+    """Weights of one det-sample; hwp_angle None = no HWP (then gamma has no effect, reading R3)."""
     q = _arr(q, np.float64); w = np.zeros(3)
     eta = (1.0 - epsilon) / (1.0 + epsilon)
-    lib().oracle_stokes_iqu(_p(q), hwp_angle, eta, cal, _p(w))
+    lib().oracle_stokes_iqu_ex(_p(q), int(hwp_angle is not None), 0.0 if hwp_angle is None else float(hwp_angle),
+                               float(gamma), int(bool(iau)), eta, cal, _p(w))
     return w
 
 
-def det_sample_probe(fp_q, bore_q, hwp_angle, epsilon, cal, flagged, nside, nest):
-    """One det-sample through A1->A2->A3: returns (pix, weights[3], dir[3])."""
+def det_sample_probe(fp_q, bore_q, hwp_angle, epsilon, cal, flagged, nside, nest, gamma=0.0, iau=False):
+    """One det-sample through A1->A2->A3: returns (pix, weights[3], dir[3]).  hwp_angle None = no
+    HWP (identical to 0.0 unless gamma != 0, reading R3)."""
     fp_q = _arr(fp_q, np.float64); bore_q = _arr(bore_q, np.float64)
     pix = np.zeros(1, np.int64); w = np.zeros(3); d = np.zeros(3)
-    lib().oracle_det_sample_probe(_p(fp_q), _p(bore_q), float(hwp_angle), float(epsilon), float(cal),
-                                  int(bool(flagged)), nside, int(nest), _p(pix), _p(w), _p(d))
+    lib().oracle_det_sample_probe_ex(_p(fp_q), _p(bore_q), int(hwp_angle is not None),
+                                     0.0 if hwp_angle is None else float(hwp_angle), float(gamma), int(bool(iau)),
+                                     float(epsilon), float(cal), int(bool(flagged)), nside, int(nest), _p(pix), _p(w),
+                                     _p(d))
     return int(pix[0]), w, d
 
 
@@ -183,16 +195,17 @@ def pixels_healpix(quats, intervals, nside, nest, n_pix_submap, shared_flags=Non
 
 
 def stokes_weights_iqu(quats, intervals, epsilon, cal, hwp=None, quat_index=None, weight_index=None,
-                       weights=None, n_det=None):
+                       weights=None, n_det=None, gamma=None, iau=False):
     quats = _arr(quats, np.float64)
     n_samp = quats.shape[1]
     n_det = n_det if n_det is not None else quats.shape[0]
     iv = intervals_array(intervals) if not isinstance(intervals, np.ndarray) else intervals
     if weights is None:
         weights = np.zeros((n_det, n_samp, 3))
-    lib().oracle_stokes_weights_iqu(_p(_arr(quat_index, np.int32)), _p(quats), _p(_arr(weight_index, np.int32)),
-                                    _p(weights), _p(_arr(hwp, np.float64)), _p(_arr(epsilon, np.float64)),
-                                    float(cal), _p(iv), len(iv), n_det, n_samp)
+    lib().oracle_stokes_weights_iqu_ex(_p(_arr(quat_index, np.int32)), _p(quats), _p(_arr(weight_index, np.int32)),
+                                       _p(weights), _p(_arr(hwp, np.float64)), _p(_arr(epsilon, np.float64)),
+                                       _p(_arr(gamma, np.float64)), int(bool(iau)), float(cal), _p(iv), len(iv),
+                                       n_det, n_samp)
     return weights
 
 
@@ -234,7 +247,7 @@ def scan_map(mapdata, global2local, n_pix_submap, pixels, weights, det_data, int
 def pointing_to_map(fp_quats, boresight, epsilon, cal, det_scale, det_data, intervals, nside, nest, nnz,
                     global2local, n_pix_submap, zmap=None, hwp=None, det_flags=None, det_flag_mask=0,
                     shared_flags=None, shared_flag_mask=0, hit_submaps=None, pixels_out=None, weights_out=None,
-                    absmap=None):
+                    absmap=None, gamma=None, iau=False):
     fp = _arr(fp_quats, np.float64); bore = _arr(boresight, np.float64)
     det_data = _arr(det_data, np.float64)
     n_det, n_samp = fp.shape[0], bore.shape[0]
@@ -242,12 +255,12 @@ def pointing_to_map(fp_quats, boresight, epsilon, cal, det_scale, det_data, inte
     g2l = _arr(global2local, np.int64)
     if zmap is None:
         zmap = np.zeros((int(g2l.max()) + 1, n_pix_submap, nnz))
-    lib().oracle_pointing_to_map(_p(fp), _p(bore), _p(_arr(hwp, np.float64)), _p(_arr(epsilon, np.float64)),
-                                 float(cal), _p(_arr(det_scale, np.float64)), _p(det_data),
-                                 _p(_arr(det_flags, np.uint8)), det_flag_mask, _p(_arr(shared_flags, np.uint8)),
-                                 shared_flag_mask, _p(iv), len(iv), nside, int(nest), nnz, _p(g2l), n_pix_submap,
-                                 _p(zmap), _p(hit_submaps), _p(pixels_out), _p(weights_out), n_det, n_samp,
-                                 _p(absmap))
+    lib().oracle_pointing_to_map_ex(_p(fp), _p(bore), _p(_arr(hwp, np.float64)), _p(_arr(epsilon, np.float64)),
+                                    float(cal), _p(_arr(det_scale, np.float64)), _p(det_data),
+                                    _p(_arr(det_flags, np.uint8)), det_flag_mask, _p(_arr(shared_flags, np.uint8)),
+                                    shared_flag_mask, _p(iv), len(iv), nside, int(nest), nnz, _p(g2l), n_pix_submap,
+                                    _p(zmap), _p(hit_submaps), _p(pixels_out), _p(weights_out), n_det, n_samp,
+                                    _p(absmap), _p(_arr(gamma, np.float64)), int(bool(iau)))
     return zmap
 
 
@@ -268,17 +281,18 @@ def pointing_to_map_omp(fp_quats, boresight, epsilon, cal, det_scale, det_data, 
 
 def pointing_to_tod(fp_quats, boresight, epsilon, cal, intervals, nside, nest, nnz, global2local, n_pix_submap,
                     mapdata, det_data, data_scale=1.0, should_zero=False, should_subtract=False, hwp=None,
-                    shared_flags=None, shared_flag_mask=0, bscale=None):
+                    shared_flags=None, shared_flag_mask=0, bscale=None, gamma=None, iau=False):
     """f1: A1 -> A2 -> A3 -> A5 per det-sample (scan a map onto the timestream in place)."""
     fp = _arr(fp_quats, np.float64); bore = _arr(boresight, np.float64)
     n_det, n_samp = fp.shape[0], bore.shape[0]
     iv = intervals_array(intervals) if not isinstance(intervals, np.ndarray) else intervals
     assert det_data.dtype == np.float64 and det_data.flags["C_CONTIGUOUS"] and det_data.shape == (n_det, n_samp)
-    lib().oracle_pointing_to_tod(_p(fp), _p(bore), _p(_arr(hwp, np.float64)), _p(_arr(epsilon, np.float64)),
-                                 float(cal), _p(_arr(shared_flags, np.uint8)), shared_flag_mask, _p(iv), len(iv),
-                                 nside, int(nest), nnz, _p(_arr(global2local, np.int64)), n_pix_submap,
-                                 _p(_arr(mapdata, np.float64)), float(data_scale), int(should_zero),
-                                 int(should_subtract), _p(det_data), n_det, n_samp, _p(bscale))
+    lib().oracle_pointing_to_tod_ex(_p(fp), _p(bore), _p(_arr(hwp, np.float64)), _p(_arr(epsilon, np.float64)),
+                                    float(cal), _p(_arr(shared_flags, np.uint8)), shared_flag_mask, _p(iv), len(iv),
+                                    nside, int(nest), nnz, _p(_arr(global2local, np.int64)), n_pix_submap,
+                                    _p(_arr(mapdata, np.float64)), float(data_scale), int(should_zero),
+                                    int(should_subtract), _p(det_data), n_det, n_samp, _p(bscale),
+                                    _p(_arr(gamma, np.float64)), int(bool(iau)))
     return det_data
 
 

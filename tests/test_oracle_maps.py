@@ -247,3 +247,63 @@ def test_pointing_to_tod_constant_map_and_adjoint(small):
                            shared_flag_mask=w.shared_flag_mask)
     lhs, rhs = float(np.sum(scanned * t)), float(np.sum(z * m))
     assert abs(lhs - rhs) <= 1e-12 * (float(np.sum(np.abs(scanned * t))) + 1.0)
+
+
+@pytest.mark.parametrize("variant", ["plain", "gamma_iau"])
+def test_det_sample_probe_equals_fused_outputs(variant):
+    """oracle.det_sample_probe (the one-by-one expectation of the full-size parity tests and the
+    direction fed to the T1 classifier) is pinned to the fused oracle's debug outputs and to the
+    A1 composition: pixel and weights element by element, direction == R(q_det) z with q_det
+    from oracle.pointing_detector; shared-flagged samples give pixel -1."""
+    w = synth.make_workload("c2", n_det=4, n_samp=300_000, nside=64)  # long enough for the 0x02 bursts
+    gamma = np.linspace(-1.0, 1.0, w.n_det) if variant == "gamma_iau" else None
+    iau = variant == "gamma_iau"
+    smask = w.shared_flag_mask | 2  # the 0x02 bursts lie inside intervals: flagged in-interval samples
+    pix = np.full((w.n_det, w.n_samp), -7, np.int64)
+    wts = np.zeros((w.n_det, w.n_samp, 3))
+    oracle.pointing_to_map(w.fp_quats, w.boresight, w.epsilon, w.cal, w.det_scale, w.det_data, w.intervals, w.nside,
+                           w.nest, 3, w.global2local, w.n_pix_submap, hwp=w.hwp, det_flags=w.det_flags,
+                           det_flag_mask=w.det_flag_mask, shared_flags=w.shared_flags,
+                           shared_flag_mask=smask, pixels_out=pix, weights_out=wts, gamma=gamma, iau=iau)
+    quats = oracle.pointing_detector(w.fp_quats, w.boresight, w.intervals, w.shared_flags, smask)
+    rng = np.random.default_rng(7)
+    inside = np.nonzero(_mask_intervals(w.intervals, w.n_samp))[0]
+    flagged_in = inside[(w.shared_flags[inside] & smask) != 0]
+    samples = np.concatenate([rng.choice(inside, 400), flagged_in[:50]])
+    n_flagged = 0
+    for s in samples:
+        d = int(rng.integers(w.n_det))
+        fl = bool(w.shared_flags[s] & smask)
+        p, wt, v = oracle.det_sample_probe(w.fp_quats[d], w.boresight[s], w.hwp[s], w.epsilon[d], w.cal, fl, w.nside,
+                                           w.nest, gamma=0.0 if gamma is None else gamma[d], iau=iau)
+        assert p == pix[d, s]
+        np.testing.assert_array_equal(wt, wts[d, s])
+        np.testing.assert_array_equal(v, oracle.quat_rotate(quats[d, s], [0.0, 0.0, 1.0]))
+        if fl:
+            assert p == -1
+            n_flagged += 1
+        else:
+            assert p == oracle.vec2pix(w.nside, w.nest, v)
+    assert n_flagged > 10
+
+
+def test_fused_gamma_iau_equals_composition(small):
+    """The fused oracle with the reading-R3 variant equals A1 -> A2 -> A3(gamma, IAU) -> A4."""
+    w = small
+    gamma = np.linspace(-0.7, 0.9, w.n_det)
+    quats = oracle.pointing_detector(w.fp_quats, w.boresight, w.intervals, w.shared_flags, w.shared_flag_mask)
+    pix, _ = oracle.pixels_healpix(quats, w.intervals, w.nside, w.nest, w.n_pix_submap, w.shared_flags,
+                                   w.shared_flag_mask)
+    wts = oracle.stokes_weights_iqu(quats, w.intervals, w.epsilon, w.cal, hwp=w.hwp, gamma=gamma, iau=True)
+    wts_plain = oracle.stokes_weights_iqu(quats, w.intervals, w.epsilon, w.cal, hwp=w.hwp)
+    m = _mask_intervals(w.intervals, w.n_samp)
+    assert np.abs(wts[:, m, 1:] - wts_plain[:, m, 1:]).max() > 0.1  # the variant changes Q/U
+    z1 = np.zeros((w.n_submap, w.n_pix_submap, 3))
+    oracle.build_noise_weighted(z1, w.global2local, w.n_pix_submap, pix, wts, w.det_data, w.det_scale, w.intervals,
+                                det_flags=w.det_flags, det_flag_mask=w.det_flag_mask, shared_flags=w.shared_flags,
+                                shared_flag_mask=w.shared_flag_mask)
+    z2 = oracle.pointing_to_map(w.fp_quats, w.boresight, w.epsilon, w.cal, w.det_scale, w.det_data, w.intervals,
+                                w.nside, w.nest, 3, w.global2local, w.n_pix_submap, hwp=w.hwp, det_flags=w.det_flags,
+                                det_flag_mask=w.det_flag_mask, shared_flags=w.shared_flags,
+                                shared_flag_mask=w.shared_flag_mask, gamma=gamma, iau=True)
+    np.testing.assert_array_equal(z2, z1)

@@ -83,3 +83,91 @@ def test_epsilon_limits():
     assert w1[0] == 1.7 and w1[1] == 0.0 and w1[2] == 0.0
     w0 = oracle.stokes_iqu(q, 0.3, 0.0, 1.0)
     assert abs(math.hypot(w0[1], w0[2]) - 1.0) < 1e-15
+
+
+# ----------------------------------------------------------------------------- reading R3 (f4)
+
+def _mueller_response(psi, hwp_axis):
+    """Detector response row (I, Q, U) of a linear polariser at sky angle psi behind an ideal
+    half-wave plate with its fast axis at sky angle hwp_axis — Mueller calculus, written
+    from the textbook matrices (polariser row 1/2 [1, cos 2psi, sin 2psi]; HWP at angle a:
+    [[1, 0, 0], [0, cos 4a, sin 4a], [0, sin 4a, -cos 4a]] on (I, Q, U)), normalised to I = 1."""
+    pol = np.array([1.0, math.cos(2 * psi), math.sin(2 * psi)])
+    if hwp_axis is None:
+        return pol
+    c, s = math.cos(4 * hwp_axis), math.sin(4 * hwp_axis)
+    hwp = np.array([[1.0, 0.0, 0.0], [0.0, c, s], [0.0, s, -c]])
+    return pol @ hwp
+
+
+def test_gamma_hwp_convention_matches_mueller_calculus():
+    """Reading R3: with an HWP at angle chi from the focal-plane x axis and a detector at angle
+    gamma in the focal plane, the HWP fast axis lies at psi - gamma + chi on the sky; the
+    Mueller response of that system is (1, cos(2 psi + 4 (chi - gamma)), sin(...))."""
+    rng = np.random.default_rng(16)
+    n = 0
+    for _ in range(400):
+        ax, a = random_axis_angle(rng)
+        r = rodrigues(ax, a)
+        d, o = r[:, 2], r[:, 0]
+        if math.hypot(d[0], d[1]) < 1e-3:
+            continue
+        psi = psi_geometric(d, o)
+        chi, gamma = rng.uniform(0, 2 * math.pi), rng.uniform(-math.pi, math.pi)
+        eps, cal = rng.uniform(0, 0.1), rng.uniform(0.5, 2.0)
+        eta = (1 - eps) / (1 + eps)
+        want = _mueller_response(psi, psi - gamma + chi) * np.array([cal, eta * cal, eta * cal])
+        got = oracle.stokes_iqu(axis_angle_quat(ax, a), chi, eps, cal, gamma=gamma)
+        np.testing.assert_allclose(got, want, atol=2e-13)
+        # without an HWP the detector angle is already inside the quaternion: gamma has no effect
+        want0 = _mueller_response(psi, None) * np.array([cal, eta * cal, eta * cal])
+        np.testing.assert_allclose(oracle.stokes_iqu(axis_angle_quat(ax, a), None, eps, cal, gamma=gamma), want0,
+                                   atol=2e-13)
+        n += 1
+    assert n > 350
+
+
+def test_iau_flips_u_only():
+    rng = np.random.default_rng(17)
+    for _ in range(200):
+        q = axis_angle_quat(*random_axis_angle(rng))
+        chi = rng.uniform(0, 2 * math.pi) if rng.random() < 0.5 else None
+        g = rng.uniform(-1, 1)
+        w = oracle.stokes_iqu(q, chi, 0.01, 1.3, gamma=g)
+        wi = oracle.stokes_iqu(q, chi, 0.01, 1.3, gamma=g, iau=True)
+        assert wi[0] == w[0] and wi[1] == w[1] and wi[2] == -w[2]
+
+
+def test_gamma_zero_and_hwp_zero_reduce_to_plain_reading():
+    """gamma = 0 is reading S9 exactly; an HWP angle of 0 equals no HWP when gamma = 0."""
+    rng = np.random.default_rng(18)
+    for _ in range(100):
+        q = axis_angle_quat(*random_axis_angle(rng))
+        chi = rng.uniform(0, 2 * math.pi)
+        np.testing.assert_array_equal(oracle.stokes_iqu(q, chi, 0.02, 1.0),
+                                      oracle.stokes_iqu(q, chi, 0.02, 1.0, gamma=0.0))
+        np.testing.assert_array_equal(oracle.stokes_iqu(q, 0.0, 0.02, 1.0), oracle.stokes_iqu(q, None, 0.02, 1.0))
+
+
+def test_unwrapped_hwp_angle_is_exact_to_the_angle():
+    """Reading R1: an unwrapped HWP angle (a 2 Hz HWP over days: chi ~ 1e6 rad) still gives the
+    response of the exact angle 2 psi + 4 chi (evaluated here in 60-digit arithmetic from the
+    geometric psi), not that of the rounded fp64 sum, which is off by up to |4 chi| 2^-53."""
+    import mpmath
+    mpmath.mp.dps = 60
+    rng = np.random.default_rng(19)
+    worst_sum = 0.0
+    for _ in range(200):
+        ax, a = random_axis_angle(rng)
+        r = rodrigues(ax, a)
+        d, o = r[:, 2], r[:, 0]
+        if math.hypot(d[0], d[1]) < 1e-2:
+            continue
+        psi = psi_geometric(d, o)
+        chi = float(rng.uniform(1e5, 4e6))
+        ang = 2 * mpmath.mpf(psi) + 4 * mpmath.mpf(chi)
+        want = [1.0, float(mpmath.cos(ang)), float(mpmath.sin(ang))]
+        got = oracle.stokes_iqu(axis_angle_quat(ax, a), chi, 0.0, 1.0)
+        np.testing.assert_allclose(got, want, atol=2e-13)
+        worst_sum = max(worst_sum, abs(math.cos(2 * psi + 4 * chi) - want[1]))
+    assert worst_sum > 1e-11  # the naive fp64 sum would not pass this pin
