@@ -77,7 +77,7 @@ def _declare(L):
     L.oracle_pointing_to_map.argtypes = [P, P, P, P, D, P, P, P, U8, P, U8, P, I64, I64, INT, I64, P, I64, P, P,
                                          P, P, I64, I64, P]
     L.oracle_pointing_to_map_ex.argtypes = [P, P, P, P, D, P, P, P, U8, P, U8, P, I64, I64, INT, I64, P, I64, P,
-                                            P, P, P, I64, I64, P, P, INT]
+                                            P, P, P, I64, I64, P, P, INT, P]
     L.oracle_pointing_to_map_omp.argtypes = [P, P, P, P, D, P, P, P, U8, P, U8, P, I64, I64, INT, I64, P, I64,
                                              P, I64, I64, INT]
     L.oracle_pointing_to_map_omp.restype = INT
@@ -247,7 +247,9 @@ def scan_map(mapdata, global2local, n_pix_submap, pixels, weights, det_data, int
 def pointing_to_map(fp_quats, boresight, epsilon, cal, det_scale, det_data, intervals, nside, nest, nnz,
                     global2local, n_pix_submap, zmap=None, hwp=None, det_flags=None, det_flag_mask=0,
                     shared_flags=None, shared_flag_mask=0, hit_submaps=None, pixels_out=None, weights_out=None,
-                    absmap=None, gamma=None, iau=False):
+                    absmap=None, gamma=None, iau=False, t2map=None):
+    """A6.  absmap (optional, zmap's shape) += |terms| (T4 scale); t2map (optional) += the T2
+    weight tolerance of each Q/U term propagated through |det_scale tod| (T4)."""
     fp = _arr(fp_quats, np.float64); bore = _arr(boresight, np.float64)
     det_data = _arr(det_data, np.float64)
     n_det, n_samp = fp.shape[0], bore.shape[0]
@@ -260,7 +262,7 @@ def pointing_to_map(fp_quats, boresight, epsilon, cal, det_scale, det_data, inte
                                     _p(_arr(det_flags, np.uint8)), det_flag_mask, _p(_arr(shared_flags, np.uint8)),
                                     shared_flag_mask, _p(iv), len(iv), nside, int(nest), nnz, _p(g2l), n_pix_submap,
                                     _p(zmap), _p(hit_submaps), _p(pixels_out), _p(weights_out), n_det, n_samp,
-                                    _p(absmap), _p(_arr(gamma, np.float64)), int(bool(iau)))
+                                    _p(absmap), _p(_arr(gamma, np.float64)), int(bool(iau)), _p(t2map))
     return zmap
 
 

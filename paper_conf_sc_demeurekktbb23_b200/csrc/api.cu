@@ -41,6 +41,14 @@ int cuda_fail(cudaError_t e, const char* where) {
 }
 
 // ---------------------------------------------------------------- interval work-list cache
+//
+// Work lists are cached per (device, chunk length, tail, interval set).  A new list is uploaded
+// ASYNCHRONOUSLY on the caller's stream: stream-ordered allocation (cudaMallocAsync) and a
+// cudaMemcpyAsync from a pinned host copy that the entry keeps until it is evicted, so a first
+// call is as asynchronous as every later one (and capturable in a CUDA graph).  An event recorded
+// after the upload orders launches on other streams after it.  The cache lock is held until the
+// caller's launch has been enqueued (WorkListLease), so no other host thread can evict the entry
+// in between; eviction (LRU, rare) synchronises the entry's event before freeing.
 
 struct CacheEntry {
     int device;
@@ -48,13 +56,31 @@ struct CacheEntry {
     int64_t tail;  // the last `tail` in-interval samples are cut into chunks of kTailChunk
     std::vector<toast_interval_t> intervals;
     Chunk* d_chunks;
+    Chunk* h_pinned;  // pinned staging of the upload (kept until eviction)
+    cudaEvent_t uploaded;
+    cudaStream_t upload_stream;
     int64_t n_chunks;
     int64_t n_samples;
+    uint64_t last_use;
 };
 
 std::mutex g_cache_mu;
 std::vector<CacheEntry> g_cache;
-constexpr size_t kCacheMax = 64;
+uint64_t g_cache_clock = 0;
+constexpr size_t kCacheMax = 256;
+
+void free_entry(CacheEntry& c) {
+    int cur = 0;
+    cudaGetDevice(&cur);
+    cudaSetDevice(c.device);
+    if (c.uploaded) {
+        cudaEventSynchronize(c.uploaded);
+        cudaEventDestroy(c.uploaded);
+    }
+    if (c.d_chunks) cudaFree(c.d_chunks);
+    if (c.h_pinned) cudaFreeHost(c.h_pinned);
+    cudaSetDevice(cur);
+}
 
 int validate_intervals(const toast_interval_t* iv, int64_t n, int64_t n_samp) {
     if (n < 0) return fail(TOAST_EINVAL, "n_intervals < 0");
@@ -70,7 +96,6 @@ int validate_intervals(const toast_interval_t* iv, int64_t n, int64_t n_samp) {
     return TOAST_OK;
 }
 
-// Returns the device work list for these intervals (creating it on first use).
 // Chunk length of the work-list tail (see fused_worklist).
 #ifndef TB_TAIL_CHUNK
 #define TB_TAIL_CHUNK 32
@@ -80,21 +105,17 @@ int validate_intervals(const toast_interval_t* iv, int64_t n, int64_t n_samp) {
 #endif
 constexpr int kTailChunk = TB_TAIL_CHUNK;
 
-int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, WorkList* out, int chunk = kChunk,
-                 int64_t tail = 0) {
-    int rc = validate_intervals(iv, n, n_samp);
-    if (rc != TOAST_OK) return rc;
-    int dev = 0;
-    cudaError_t e = cudaGetDevice(&dev);
-    if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
-    std::lock_guard<std::mutex> lk(g_cache_mu);
-    for (auto& c : g_cache) {
-        if (c.device == dev && c.chunk == chunk && c.tail == tail && (int64_t)c.intervals.size() == n &&
-            (n == 0 || std::memcmp(c.intervals.data(), iv, sizeof(toast_interval_t) * n) == 0)) {
-            *out = WorkList{c.d_chunks, c.n_chunks, c.n_samples};
-            return TOAST_OK;
-        }
-    }
+// A work list valid while the lease (and so the cache lock) lives: enqueue the launch, then let
+// the lease go.
+struct WorkListLease {
+    WorkList wl;
+    std::unique_lock<std::mutex> lock;
+};
+
+// Chunks of `chunk` samples that never cross an interval and, inside an interval, end on
+// multiples of 16 samples (the fused kernel's TMA boxes), so only interval edges give partial
+// 16-sample blocks; the last `tail` in-interval samples in chunks of kTailChunk.
+std::vector<Chunk> build_chunks(const toast_interval_t* iv, int64_t n, int chunk, int64_t tail, int64_t* total_out) {
     std::vector<Chunk> chunks;
     int64_t all = 0;
     for (int64_t i = 0; i < n; ++i) all += iv[i].last - iv[i].first + 1;
@@ -102,59 +123,98 @@ int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, WorkList
     for (int64_t i = 0; i < n; ++i) {
         for (int64_t f = iv[i].first; f <= iv[i].last;) {
             const int len = (total >= all - tail) ? kTailChunk : chunk;
-            const int64_t cnt = std::min<int64_t>(len, iv[i].last - f + 1);
+            int64_t end = f + len;
+            if ((len & 15) == 0 && (end & ~int64_t(15)) > f) end &= ~int64_t(15);
+            const int64_t cnt = std::min<int64_t>(end - f, iv[i].last - f + 1);
             chunks.push_back(Chunk{f, (int32_t)cnt, (int32_t)i});
             total += cnt;
             f += cnt;
         }
     }
-    Chunk* d = nullptr;
+    *total_out = total;
+    return chunks;
+}
+
+int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, cudaStream_t st, WorkListLease* out,
+                 int chunk = kChunk, int64_t tail = 0) {
+    int rc = validate_intervals(iv, n, n_samp);
+    if (rc != TOAST_OK) return rc;
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    std::unique_lock<std::mutex> lk(g_cache_mu);
+    for (auto& c : g_cache) {
+        if (c.device == dev && c.chunk == chunk && c.tail == tail && (int64_t)c.intervals.size() == n &&
+            (n == 0 || std::memcmp(c.intervals.data(), iv, sizeof(toast_interval_t) * n) == 0)) {
+            c.last_use = ++g_cache_clock;
+            if (c.uploaded && st != c.upload_stream) {
+                e = cudaStreamWaitEvent(st, c.uploaded, 0);
+                if (e != cudaSuccess) return cuda_fail(e, "cudaStreamWaitEvent on the work-list upload");
+            }
+            out->wl = WorkList{c.d_chunks, c.n_chunks, c.n_samples};
+            out->lock = std::move(lk);
+            return TOAST_OK;
+        }
+    }
+    int64_t total = 0;
+    std::vector<Chunk> chunks = build_chunks(iv, n, chunk, tail, &total);
+    CacheEntry ce{dev, chunk, tail, std::vector<toast_interval_t>(iv, iv + n), nullptr, nullptr, nullptr, st,
+                  (int64_t)chunks.size(), total, ++g_cache_clock};
     if (!chunks.empty()) {
-        e = cudaMalloc(&d, sizeof(Chunk) * chunks.size());
+        const size_t bytes = sizeof(Chunk) * chunks.size();
+        e = cudaMallocHost(&ce.h_pinned, bytes);
         if (e != cudaSuccess) {
             cudaGetLastError();
-            return fail(TOAST_ENOMEM, "cudaMalloc of the interval work list: %s", cudaGetErrorString(e));
+            return fail(TOAST_ENOMEM, "cudaMallocHost of the work-list staging: %s", cudaGetErrorString(e));
         }
-        e = cudaMemcpy(d, chunks.data(), sizeof(Chunk) * chunks.size(), cudaMemcpyHostToDevice);
+        std::memcpy(ce.h_pinned, chunks.data(), bytes);
+        e = cudaMallocAsync(reinterpret_cast<void**>(&ce.d_chunks), bytes, st);
+        if (e == cudaSuccess) e = cudaMemcpyAsync(ce.d_chunks, ce.h_pinned, bytes, cudaMemcpyHostToDevice, st);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ce.uploaded, cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventRecord(ce.uploaded, st);
         if (e != cudaSuccess) {
-            cudaFree(d);
-            return cuda_fail(e, "cudaMemcpy of the interval work list");
+            cudaGetLastError();
+            free_entry(ce);
+            return fail(TOAST_ENOMEM, "work-list upload: %s", cudaGetErrorString(e));
         }
     }
-    if (g_cache.size() >= kCacheMax) {
-        int cur = dev;
-        cudaSetDevice(g_cache.front().device);
-        cudaFree(g_cache.front().d_chunks);
-        cudaSetDevice(cur);
-        g_cache.erase(g_cache.begin());
+    if (g_cache.size() >= kCacheMax) {  // evict the least recently used entry
+        size_t lru = 0;
+        for (size_t i = 1; i < g_cache.size(); ++i)
+            if (g_cache[i].last_use < g_cache[lru].last_use) lru = i;
+        free_entry(g_cache[lru]);
+        g_cache.erase(g_cache.begin() + (long)lru);
     }
-    g_cache.push_back(
-        CacheEntry{dev, chunk, tail, std::vector<toast_interval_t>(iv, iv + n), d, (int64_t)chunks.size(), total});
-    *out = WorkList{d, (int64_t)chunks.size(), total};
+    g_cache.push_back(std::move(ce));
+    const CacheEntry& c = g_cache.back();
+    out->wl = WorkList{c.d_chunks, c.n_chunks, c.n_samples};
+    out->lock = std::move(lk);
     return TOAST_OK;
 }
 
 // Work list of the fused kernels: chunks of kFusedChunk samples, shorter when few detector groups
 // x few samples would leave the persistent grid idle (C1: 4 detectors, one group of 32 lanes),
 // so that there are at least ~4 items per resident warp.  Items are handed out in list order,
-// so the LAST items set the kernel's tail: a warp streams one 128-sample item for ~1/6 of the
-// C2 kernel time, and warps that draw no new item idle meanwhile.  The last TB_TAIL_ITEMS items' worth of
-// samples per resident warp are therefore cut into kTailChunk-sample chunks.
-int fused_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, int64_t n_det, WorkList* out) {
-    int rc = get_worklist(iv, n, n_samp, out, kFusedChunk);
+// so the LAST items set the kernel's tail: the last TB_TAIL_ITEMS items' worth of samples per
+// resident warp are cut into kTailChunk-sample chunks.  Only the final list is built and cached.
+int fused_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, int64_t n_det, cudaStream_t st,
+                   WorkListLease* out) {
+    int rc = validate_intervals(iv, n, n_samp);
     if (rc != TOAST_OK) return rc;
+    int64_t n_samples = 0;
+    for (int64_t i = 0; i < n; ++i) n_samples += iv[i].last - iv[i].first + 1;
     const int64_t groups = (n_det + 31) / 32, warps = (int64_t)num_sms() * 16, want = 4 * warps;
     // large focal planes (>= 64 detector groups: C4, C5) take 64-sample chunks: the warps in flight
     // then span half the time window, so the map lines they scatter into are reused more in L2
-    // (measured: C5 -1.6 %; no effect below 64 groups, where the tail dominates)
     int chunk = groups >= 64 ? kFusedChunk / 2 : kFusedChunk;
-    while (chunk > 16 && (out->n_samples / chunk) * groups < want) chunk /= 2;
+    while (chunk > 16 && (n_samples / chunk) * groups < want) chunk /= 2;
 #ifndef TB_NO_TAIL
-    const int64_t tail = chunk > kTailChunk ? std::min<int64_t>(out->n_samples / 4, TB_TAIL_ITEMS * warps * kTailChunk / groups) : 0;
+    const int64_t tail =
+        chunk > kTailChunk ? std::min<int64_t>(n_samples / 4, TB_TAIL_ITEMS * warps * kTailChunk / std::max<int64_t>(groups, 1)) : 0;
 #else
     const int64_t tail = 0;
 #endif
-    return (chunk == kFusedChunk && tail == 0) ? TOAST_OK : get_worklist(iv, n, n_samp, out, chunk, tail);
+    return get_worklist(iv, n, n_samp, st, out, chunk, tail);
 }
 
 bool is_pow2(int64_t x) { return x > 0 && (x & (x - 1)) == 0; }
@@ -170,6 +230,14 @@ int check_submap(int64_t n_pix_submap, int64_t npix) {
     if (npix > 0 && npix % n_pix_submap != 0)
         return fail(TOAST_EINVAL, "n_pix_submap = %lld does not divide npix = %lld", (long long)n_pix_submap,
                     (long long)npix);
+    return TOAST_OK;
+}
+
+// The fused kernels index samples, chunks and work items with 32-bit integers.
+int check_fused_dims(int64_t n_det, int64_t n_samp) {
+    if (n_samp >= (int64_t(1) << 31))
+        return fail(TOAST_EUNSUPPORTED, "n_samp = %lld >= 2^31 in one call (split the observation)", (long long)n_samp);
+    if (n_det >= (int64_t(1) << 31)) return fail(TOAST_EUNSUPPORTED, "n_det = %lld >= 2^31", (long long)n_det);
     return TOAST_OK;
 }
 
@@ -253,15 +321,11 @@ const char* toast_version(void) { return "toastb200 0.1.0 (sm_100a)"; }
 const char* toast_last_fused_path(void) { return last_fused_path(); }
 
 int toast_release(void) {
-    std::lock_guard<std::mutex> lk(g_cache_mu);
-    int cur = 0;
-    cudaGetDevice(&cur);
-    for (auto& c : g_cache) {
-        cudaSetDevice(c.device);
-        if (c.d_chunks) cudaFree(c.d_chunks);
+    {
+        std::lock_guard<std::mutex> lk(g_cache_mu);
+        for (auto& c : g_cache) free_entry(c);
+        g_cache.clear();
     }
-    cudaSetDevice(cur);
-    g_cache.clear();
     release_offset_cache();
     return ok();
 }
@@ -276,10 +340,10 @@ int toast_pointing_detector(const double* fp_quats, const double* boresight, con
         REQUIRE(boresight);
         REQUIRE(quats);
     }
-    WorkList wl;
-    int rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    WorkListLease lease;
+    int rc = get_worklist(intervals, n_intervals, n_samp, (cudaStream_t)stream, &lease);
     if (rc != TOAST_OK) return rc;
-    cudaError_t e = launch_pointing_detector(wl, fp_quats, boresight, quat_index, quats, shared_flags,
+    cudaError_t e = launch_pointing_detector(lease.wl, fp_quats, boresight, quat_index, quats, shared_flags,
                                              shared_flag_mask, n_det, n_samp, (cudaStream_t)stream);
     if (e != cudaSuccess) return cuda_fail(e, "pointing_detector launch");
     return ok();
@@ -300,13 +364,33 @@ int toast_pixels_healpix(const int32_t* quat_index, const double* quats, const u
         REQUIRE(quats);
         REQUIRE(pixels);
     }
-    WorkList wl;
-    rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    WorkListLease lease;
+    rc = get_worklist(intervals, n_intervals, n_samp, (cudaStream_t)stream, &lease);
     if (rc != TOAST_OK) return rc;
-    cudaError_t e = launch_pixels_healpix(wl, quat_index, quats, shared_flags, shared_flag_mask, pixel_index, pixels,
+    cudaError_t e = launch_pixels_healpix(lease.wl, quat_index, quats, shared_flags, shared_flag_mask, pixel_index, pixels,
                                           hit_submaps, n_pix_submap, nside, nest, n_det, n_samp,
                                           (cudaStream_t)stream);
     if (e != cudaSuccess) return cuda_fail(e, "pixels_healpix launch");
+    return ok();
+}
+
+int toast_stokes_weights_iqu_ex(const int32_t* quat_index, const double* quats, const int32_t* weight_index,
+                                double* weights, const double* hwp, const double* epsilon, const double* gamma, int iau,
+                                double cal, const toast_interval_t* intervals, int64_t n_intervals, int64_t n_det,
+                                int64_t n_samp, void* stream) {
+    REQUIRE_DIMS(n_det, n_samp);
+    if (iau != 0 && iau != 1) return fail(TOAST_EINVAL, "iau = %d must be 0 or 1", iau);
+    if (n_det > 0 && n_intervals > 0) {
+        REQUIRE(quats);
+        REQUIRE(weights);
+        REQUIRE(epsilon);
+    }
+    WorkListLease lease;
+    int rc = get_worklist(intervals, n_intervals, n_samp, (cudaStream_t)stream, &lease);
+    if (rc != TOAST_OK) return rc;
+    cudaError_t e = launch_stokes_weights_iqu(lease.wl, quat_index, quats, weight_index, weights, hwp, epsilon, cal,
+                                              n_det, n_samp, (cudaStream_t)stream, gamma, iau);
+    if (e != cudaSuccess) return cuda_fail(e, "stokes_weights_iqu launch");
     return ok();
 }
 
@@ -314,19 +398,8 @@ int toast_stokes_weights_iqu(const int32_t* quat_index, const double* quats, con
                              double* weights, const double* hwp, const double* epsilon, double cal,
                              const toast_interval_t* intervals, int64_t n_intervals, int64_t n_det, int64_t n_samp,
                              void* stream) {
-    REQUIRE_DIMS(n_det, n_samp);
-    if (n_det > 0 && n_intervals > 0) {
-        REQUIRE(quats);
-        REQUIRE(weights);
-        REQUIRE(epsilon);
-    }
-    WorkList wl;
-    int rc = get_worklist(intervals, n_intervals, n_samp, &wl);
-    if (rc != TOAST_OK) return rc;
-    cudaError_t e = launch_stokes_weights_iqu(wl, quat_index, quats, weight_index, weights, hwp, epsilon, cal, n_det,
-                                              n_samp, (cudaStream_t)stream);
-    if (e != cudaSuccess) return cuda_fail(e, "stokes_weights_iqu launch");
-    return ok();
+    return toast_stokes_weights_iqu_ex(quat_index, quats, weight_index, weights, hwp, epsilon, nullptr, 0, cal,
+                                       intervals, n_intervals, n_det, n_samp, stream);
 }
 
 int toast_build_noise_weighted(const int64_t* global2local, double* zmap, int64_t n_pix_submap, int64_t nnz,
@@ -348,10 +421,10 @@ int toast_build_noise_weighted(const int64_t* global2local, double* zmap, int64_
         REQUIRE(det_data);
         REQUIRE(det_scale);
     }
-    WorkList wl;
-    rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    WorkListLease lease;
+    rc = get_worklist(intervals, n_intervals, n_samp, (cudaStream_t)stream, &lease);
     if (rc != TOAST_OK) return rc;
-    cudaError_t e = launch_build_noise_weighted(wl, make_map_geom(global2local, n_pix_submap), zmap, (int)nnz,
+    cudaError_t e = launch_build_noise_weighted(lease.wl, make_map_geom(global2local, n_pix_submap), zmap, (int)nnz,
                                                 pixel_index, pixels, weight_index, weights, data_index, det_data,
                                                 flag_index, det_flags, det_flag_mask, det_scale, shared_flags,
                                                 shared_flag_mask, n_det, n_samp, (cudaStream_t)stream);
@@ -375,29 +448,31 @@ int toast_scan_map(const int64_t* global2local, int64_t n_pix_submap, const doub
         REQUIRE(pixels);
         REQUIRE(weights);
     }
-    WorkList wl;
-    rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    WorkListLease lease;
+    rc = get_worklist(intervals, n_intervals, n_samp, (cudaStream_t)stream, &lease);
     if (rc != TOAST_OK) return rc;
-    cudaError_t e = launch_scan_map(wl, make_map_geom(global2local, n_pix_submap), mapdata, (int)nnz, data_index,
+    cudaError_t e = launch_scan_map(lease.wl, make_map_geom(global2local, n_pix_submap), mapdata, (int)nnz, data_index,
                                     det_data, pixel_index, pixels, weight_index, weights, data_scale, should_zero,
                                     should_subtract, n_det, n_samp, (cudaStream_t)stream);
     if (e != cudaSuccess) return cuda_fail(e, "scan_map launch");
     return ok();
 }
 
-int toast_pointing_to_map(const double* fp_quats, const double* boresight, const double* hwp, const double* epsilon,
-                          double cal, const double* det_scale, const double* det_data, const uint8_t* det_flags,
-                          uint8_t det_flag_mask, const uint8_t* shared_flags, uint8_t shared_flag_mask,
-                          const toast_interval_t* intervals, int64_t n_intervals, int64_t nside, int nest,
-                          int64_t nnz, const int64_t* global2local, int64_t n_pix_submap, double* zmap,
-                          uint8_t* hit_submaps, int64_t* pixels_out, double* weights_out, int64_t n_det,
-                          int64_t n_samp, void* stream) {
+int toast_pointing_to_map_ex(const double* fp_quats, const double* boresight, const double* hwp,
+                             const double* epsilon, double cal, const double* det_scale, const double* det_data,
+                             const uint8_t* det_flags, uint8_t det_flag_mask, const uint8_t* shared_flags,
+                             uint8_t shared_flag_mask, const toast_interval_t* intervals, int64_t n_intervals,
+                             int64_t nside, int nest, int64_t nnz, const int64_t* global2local, int64_t n_pix_submap,
+                             void* zmap, uint8_t* hit_submaps, int64_t* pixels_out, double* weights_out, int64_t n_det,
+                             int64_t n_samp, const toast_map_options_t* opts, void* stream) {
     REQUIRE_DIMS(n_det, n_samp);
     int rc = check_nside(nside);
     if (rc != TOAST_OK) return rc;
     if (nest != 0 && nest != 1) return fail(TOAST_EINVAL, "nest = %d must be 0 (RING) or 1 (NESTED)", nest);
     if (nnz != 1 && nnz != 3) return fail(TOAST_EINVAL, "nnz = %lld must be 1 or 3", (long long)nnz);
     rc = check_submap(n_pix_submap, 12 * nside * nside);
+    if (rc != TOAST_OK) return rc;
+    rc = check_fused_dims(n_det, n_samp);
     if (rc != TOAST_OK) return rc;
     if (n_det > 0 && n_intervals > 0) {
         REQUIRE(fp_quats);
@@ -408,10 +483,14 @@ int toast_pointing_to_map(const double* fp_quats, const double* boresight, const
         REQUIRE(global2local);
         REQUIRE(zmap);
     }
-    WorkList wl;
-    rc = fused_worklist(intervals, n_intervals, n_samp, n_det, &wl);
+    if (opts && opts->map_f32 && (pixels_out || weights_out))
+        return fail(TOAST_EINVAL, "debug outputs are not available with an fp32 map");
+    WorkListLease lease;
+    rc = fused_worklist(intervals, n_intervals, n_samp, n_det, (cudaStream_t)stream, &lease);
     if (rc != TOAST_OK) return rc;
-    FusedArgs a;
+    if ((int64_t)lease.wl.n_chunks * ((n_det + 31) / 32) >= (int64_t(1) << 31))
+        return fail(TOAST_EUNSUPPORTED, "more than 2^31 work items (split the call over detectors)");
+    FusedArgs a = {};
     a.fp_quats = fp_quats;
     a.boresight = boresight;
     a.hwp = hwp;
@@ -427,29 +506,48 @@ int toast_pointing_to_map(const double* fp_quats, const double* boresight, const
     a.nest = nest;
     a.nnz = (int)nnz;
     a.map = make_map_geom(global2local, n_pix_submap);
-    a.zmap = zmap;
+    a.zmap = static_cast<double*>(zmap);
     a.hit_submaps = hit_submaps;
     a.pixels_out = pixels_out;
     a.weights_out = weights_out;
     a.n_det = n_det;
     a.n_samp = n_samp;
+    if (opts) {
+        a.gamma = opts->gamma;
+        a.iau = opts->iau;
+        a.map_f32 = opts->map_f32;
+        a.dropped = opts->dropped;
+    }
     int serr = 0;
     unsigned long long* sched = sched_counter(&serr);
     if (serr) return fail(TOAST_ENOMEM, "could not allocate the work-distribution counter");
-    cudaError_t e = launch_pointing_to_map(wl, a, sched, (cudaStream_t)stream);
+    cudaError_t e = launch_pointing_to_map(lease.wl, a, sched, (cudaStream_t)stream);
     if (e != cudaSuccess) return cuda_fail(e, "pointing_to_map launch");
     return ok();
 }
 
+int toast_pointing_to_map(const double* fp_quats, const double* boresight, const double* hwp, const double* epsilon,
+                          double cal, const double* det_scale, const double* det_data, const uint8_t* det_flags,
+                          uint8_t det_flag_mask, const uint8_t* shared_flags, uint8_t shared_flag_mask,
+                          const toast_interval_t* intervals, int64_t n_intervals, int64_t nside, int nest,
+                          int64_t nnz, const int64_t* global2local, int64_t n_pix_submap, double* zmap,
+                          uint8_t* hit_submaps, int64_t* pixels_out, double* weights_out, int64_t n_det,
+                          int64_t n_samp, void* stream) {
+    return toast_pointing_to_map_ex(fp_quats, boresight, hwp, epsilon, cal, det_scale, det_data, det_flags,
+                                    det_flag_mask, shared_flags, shared_flag_mask, intervals, n_intervals, nside, nest,
+                                    nnz, global2local, n_pix_submap, zmap, hit_submaps, pixels_out, weights_out, n_det,
+                                    n_samp, nullptr, stream);
+}
+
 }  // extern "C"
 
-extern "C" int toast_pointing_to_tod(const double* fp_quats, const double* boresight, const double* hwp,
-                                     const double* epsilon, double cal, const uint8_t* shared_flags,
-                                     uint8_t shared_flag_mask, const toast_interval_t* intervals, int64_t n_intervals,
-                                     int64_t nside, int nest, int64_t nnz, const int64_t* global2local,
-                                     int64_t n_pix_submap, const double* mapdata, double data_scale, int should_zero,
-                                     int should_subtract, double* det_data, int64_t n_det, int64_t n_samp,
-                                     void* stream) {
+extern "C" int toast_pointing_to_tod_ex(const double* fp_quats, const double* boresight, const double* hwp,
+                                        const double* epsilon, double cal, const uint8_t* shared_flags,
+                                        uint8_t shared_flag_mask, const toast_interval_t* intervals,
+                                        int64_t n_intervals, int64_t nside, int nest, int64_t nnz,
+                                        const int64_t* global2local, int64_t n_pix_submap, const void* mapdata,
+                                        double data_scale, int should_zero, int should_subtract, double* det_data,
+                                        int64_t n_det, int64_t n_samp, const toast_map_options_t* opts, void* stream) {
     using namespace toastb200;
     REQUIRE_DIMS(n_det, n_samp);
     int rc = check_nside(nside);
@@ -457,6 +555,8 @@ extern "C" int toast_pointing_to_tod(const double* fp_quats, const double* bores
     if (nest != 0 && nest != 1) return fail(TOAST_EINVAL, "nest = %d must be 0 (RING) or 1 (NESTED)", nest);
     if (nnz != 1 && nnz != 3) return fail(TOAST_EINVAL, "nnz = %lld must be 1 or 3", (long long)nnz);
     rc = check_submap(n_pix_submap, 12 * nside * nside);
+    if (rc != TOAST_OK) return rc;
+    rc = check_fused_dims(n_det, n_samp);
     if (rc != TOAST_OK) return rc;
     if (n_det > 0 && n_intervals > 0) {
         REQUIRE(fp_quats);
@@ -466,9 +566,12 @@ extern "C" int toast_pointing_to_tod(const double* fp_quats, const double* bores
         REQUIRE(mapdata);
         REQUIRE(det_data);
     }
-    WorkList wl;
-    rc = fused_worklist(intervals, n_intervals, n_samp, n_det, &wl);
+    if (opts && opts->dropped) return fail(TOAST_EINVAL, "the dropped-sample counter applies to pointing_to_map only");
+    WorkListLease lease;
+    rc = fused_worklist(intervals, n_intervals, n_samp, n_det, (cudaStream_t)stream, &lease);
     if (rc != TOAST_OK) return rc;
+    if ((int64_t)lease.wl.n_chunks * ((n_det + 31) / 32) >= (int64_t(1) << 31))
+        return fail(TOAST_EUNSUPPORTED, "more than 2^31 work items (split the call over detectors)");
     FusedArgs a = {};
     a.fp_quats = fp_quats;
     a.boresight = boresight;
@@ -485,17 +588,34 @@ extern "C" int toast_pointing_to_tod(const double* fp_quats, const double* bores
     a.map = make_map_geom(global2local, n_pix_submap);
     a.n_det = n_det;
     a.n_samp = n_samp;
-    a.mapdata = mapdata;
+    a.mapdata = static_cast<const double*>(mapdata);
     a.data_scale = data_scale;
     a.should_zero = should_zero;
     a.should_subtract = should_subtract;
     a.tod_out = det_data;
+    if (opts) {
+        a.gamma = opts->gamma;
+        a.iau = opts->iau;
+        a.map_f32 = opts->map_f32;
+    }
     int serr = 0;
     unsigned long long* sched = sched_counter(&serr);
     if (serr) return fail(TOAST_ENOMEM, "could not allocate the work-distribution counter");
-    cudaError_t e = launch_pointing_to_tod(wl, a, sched, (cudaStream_t)stream);
+    cudaError_t e = launch_pointing_to_tod(lease.wl, a, sched, (cudaStream_t)stream);
     if (e != cudaSuccess) return cuda_fail(e, "pointing_to_tod launch");
     return ok();
+}
+
+extern "C" int toast_pointing_to_tod(const double* fp_quats, const double* boresight, const double* hwp,
+                                     const double* epsilon, double cal, const uint8_t* shared_flags,
+                                     uint8_t shared_flag_mask, const toast_interval_t* intervals, int64_t n_intervals,
+                                     int64_t nside, int nest, int64_t nnz, const int64_t* global2local,
+                                     int64_t n_pix_submap, const double* mapdata, double data_scale, int should_zero,
+                                     int should_subtract, double* det_data, int64_t n_det, int64_t n_samp,
+                                     void* stream) {
+    return toast_pointing_to_tod_ex(fp_quats, boresight, hwp, epsilon, cal, shared_flags, shared_flag_mask, intervals,
+                                    n_intervals, nside, nest, nnz, global2local, n_pix_submap, mapdata, data_scale,
+                                    should_zero, should_subtract, det_data, n_det, n_samp, nullptr, stream);
 }
 
 // ---------------------------------------------------------------- NEXT rows (f2, f4)
@@ -508,52 +628,87 @@ struct OffsetCacheEntry {
     int step;
     std::vector<toast_interval_t> intervals;
     int64_t* d_arrays;  // [2][n]: iv_first, view_base
+    int64_t* h_pinned;  // pinned staging of the upload (kept until eviction)
+    cudaEvent_t uploaded;
+    cudaStream_t upload_stream;
+    uint64_t last_use;
 };
 std::mutex g_ocache_mu;
 std::vector<OffsetCacheEntry> g_ocache;
+uint64_t g_ocache_clock = 0;
 
-int get_offset_views(const toast_interval_t* iv, int64_t n, int64_t step, OffsetViews* out) {
+void free_oentry(OffsetCacheEntry& c) {
+    int cur = 0;
+    cudaGetDevice(&cur);
+    cudaSetDevice(c.device);
+    if (c.uploaded) {
+        cudaEventSynchronize(c.uploaded);
+        cudaEventDestroy(c.uploaded);
+    }
+    if (c.d_arrays) cudaFree(c.d_arrays);
+    if (c.h_pinned) cudaFreeHost(c.h_pinned);
+    cudaSetDevice(cur);
+}
+
+// Offset views of an interval set, uploaded asynchronously on the caller's stream like the work
+// lists (the lock is held through the caller's launch by the lease).
+int get_offset_views(const toast_interval_t* iv, int64_t n, int64_t step, cudaStream_t st, OffsetViews* out,
+                     std::unique_lock<std::mutex>* lease) {
     if (step < 1 || step > (int64_t(1) << 30)) return fail(TOAST_EINVAL, "step_length = %lld must be in [1, 2^30]",
                                                            (long long)step);
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
-    std::lock_guard<std::mutex> lk(g_ocache_mu);
+    std::unique_lock<std::mutex> lk(g_ocache_mu);
     for (auto& c : g_ocache) {
         if (c.device == dev && c.step == (int)step && (int64_t)c.intervals.size() == n &&
             (n == 0 || std::memcmp(c.intervals.data(), iv, sizeof(toast_interval_t) * n) == 0)) {
+            c.last_use = ++g_ocache_clock;
+            if (c.uploaded && st != c.upload_stream) {
+                e = cudaStreamWaitEvent(st, c.uploaded, 0);
+                if (e != cudaSuccess) return cuda_fail(e, "cudaStreamWaitEvent on the offset-view upload");
+            }
             *out = OffsetViews{c.d_arrays, c.d_arrays + n, (int)step};
+            *lease = std::move(lk);
             return TOAST_OK;
         }
     }
-    std::vector<int64_t> h(2 * std::max<int64_t>(n, 1), 0);
+    const size_t cnt = 2 * (size_t)std::max<int64_t>(n, 1);
+    OffsetCacheEntry ce{dev, (int)step, std::vector<toast_interval_t>(iv, iv + n), nullptr, nullptr, nullptr, st,
+                        ++g_ocache_clock};
+    e = cudaMallocHost(&ce.h_pinned, sizeof(int64_t) * cnt);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(TOAST_ENOMEM, "cudaMallocHost of the offset views: %s", cudaGetErrorString(e));
+    }
     int64_t base = 0;
+    ce.h_pinned[0] = ce.h_pinned[cnt - 1] = 0;
     for (int64_t i = 0; i < n; ++i) {
-        h[i] = iv[i].first;
-        h[n + i] = base;
+        ce.h_pinned[i] = iv[i].first;
+        ce.h_pinned[n + i] = base;
         const int64_t len = iv[i].last - iv[i].first + 1;
         base += (len + step - 1) / step;
     }
-    int64_t* d = nullptr;
-    e = cudaMalloc(&d, sizeof(int64_t) * h.size());
+    e = cudaMallocAsync(reinterpret_cast<void**>(&ce.d_arrays), sizeof(int64_t) * cnt, st);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(ce.d_arrays, ce.h_pinned, sizeof(int64_t) * cnt, cudaMemcpyHostToDevice, st);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ce.uploaded, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventRecord(ce.uploaded, st);
     if (e != cudaSuccess) {
         cudaGetLastError();
-        return fail(TOAST_ENOMEM, "cudaMalloc of the offset views: %s", cudaGetErrorString(e));
-    }
-    e = cudaMemcpy(d, h.data(), sizeof(int64_t) * h.size(), cudaMemcpyHostToDevice);
-    if (e != cudaSuccess) {
-        cudaFree(d);
-        return cuda_fail(e, "cudaMemcpy of the offset views");
+        free_oentry(ce);
+        return fail(TOAST_ENOMEM, "offset-view upload: %s", cudaGetErrorString(e));
     }
     if (g_ocache.size() >= kCacheMax) {
-        int cur = dev;
-        cudaSetDevice(g_ocache.front().device);
-        cudaFree(g_ocache.front().d_arrays);
-        cudaSetDevice(cur);
-        g_ocache.erase(g_ocache.begin());
+        size_t lru = 0;
+        for (size_t i = 1; i < g_ocache.size(); ++i)
+            if (g_ocache[i].last_use < g_ocache[lru].last_use) lru = i;
+        free_oentry(g_ocache[lru]);
+        g_ocache.erase(g_ocache.begin() + (long)lru);
     }
-    g_ocache.push_back(OffsetCacheEntry{dev, (int)step, std::vector<toast_interval_t>(iv, iv + n), d});
-    *out = OffsetViews{d, d + n, (int)step};
+    g_ocache.push_back(std::move(ce));
+    const OffsetCacheEntry& c = g_ocache.back();
+    *out = OffsetViews{c.d_arrays, c.d_arrays + n, (int)step};
+    *lease = std::move(lk);
     return TOAST_OK;
 }
 
@@ -561,13 +716,7 @@ int get_offset_views(const toast_interval_t* iv, int64_t n, int64_t step, Offset
 
 void release_offset_cache() {
     std::lock_guard<std::mutex> lk(g_ocache_mu);
-    int cur = 0;
-    cudaGetDevice(&cur);
-    for (auto& c : g_ocache) {
-        cudaSetDevice(c.device);
-        cudaFree(c.d_arrays);
-    }
-    cudaSetDevice(cur);
+    for (auto& c : g_ocache) free_oentry(c);
     g_ocache.clear();
 }
 
@@ -579,10 +728,10 @@ extern "C" int toast_stokes_weights_i(const int32_t* weight_index, double* weigh
     using namespace toastb200;
     REQUIRE_DIMS(n_det, n_samp);
     if (n_det > 0 && n_intervals > 0) REQUIRE(weights);
-    WorkList wl;
-    int rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    WorkListLease lease;
+    int rc = get_worklist(intervals, n_intervals, n_samp, (cudaStream_t)stream, &lease);
     if (rc != TOAST_OK) return rc;
-    cudaError_t e = launch_stokes_weights_i(wl, weight_index, weights, cal, n_det, n_samp, (cudaStream_t)stream);
+    cudaError_t e = launch_stokes_weights_i(lease.wl, weight_index, weights, cal, n_det, n_samp, (cudaStream_t)stream);
     if (e != cudaSuccess) return cuda_fail(e, "stokes_weights_i launch");
     return ok();
 }
@@ -596,10 +745,10 @@ extern "C" int toast_noise_weight(const int32_t* data_index, double* det_data, c
         REQUIRE(det_data);
         REQUIRE(det_weights);
     }
-    WorkList wl;
-    int rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    WorkListLease lease;
+    int rc = get_worklist(intervals, n_intervals, n_samp, (cudaStream_t)stream, &lease);
     if (rc != TOAST_OK) return rc;
-    cudaError_t e = launch_noise_weight(wl, data_index, det_data, det_weights, n_det, n_samp, (cudaStream_t)stream);
+    cudaError_t e = launch_noise_weight(lease.wl, data_index, det_data, det_weights, n_det, n_samp, (cudaStream_t)stream);
     if (e != cudaSuccess) return cuda_fail(e, "noise_weight launch");
     return ok();
 }
@@ -615,13 +764,14 @@ extern "C" int toast_template_offset_add_to_signal(int64_t step_length, const in
         REQUIRE(amplitudes);
         REQUIRE(det_data);
     }
-    WorkList wl;
-    int rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    WorkListLease lease;
+    int rc = get_worklist(intervals, n_intervals, n_samp, (cudaStream_t)stream, &lease);
     if (rc != TOAST_OK) return rc;
     OffsetViews v;
-    rc = get_offset_views(intervals, n_intervals, step_length, &v);
+    std::unique_lock<std::mutex> vlease;
+    rc = get_offset_views(intervals, n_intervals, step_length, (cudaStream_t)stream, &v, &vlease);
     if (rc != TOAST_OK) return rc;
-    cudaError_t e = launch_offset_add(wl, v, amp_offset, amplitudes, data_index, det_data, n_det, n_samp,
+    cudaError_t e = launch_offset_add(lease.wl, v, amp_offset, amplitudes, data_index, det_data, n_det, n_samp,
                                       (cudaStream_t)stream);
     if (e != cudaSuccess) return cuda_fail(e, "template_offset_add_to_signal launch");
     return ok();
@@ -639,13 +789,14 @@ extern "C" int toast_template_offset_project_signal(int64_t step_length, const i
         REQUIRE(amplitudes);
         REQUIRE(det_data);
     }
-    WorkList wl;
-    int rc = get_worklist(intervals, n_intervals, n_samp, &wl);
+    WorkListLease lease;
+    int rc = get_worklist(intervals, n_intervals, n_samp, (cudaStream_t)stream, &lease);
     if (rc != TOAST_OK) return rc;
     OffsetViews v;
-    rc = get_offset_views(intervals, n_intervals, step_length, &v);
+    std::unique_lock<std::mutex> vlease;
+    rc = get_offset_views(intervals, n_intervals, step_length, (cudaStream_t)stream, &v, &vlease);
     if (rc != TOAST_OK) return rc;
-    cudaError_t e = launch_offset_project(wl, v, amp_offset, amplitudes, data_index, det_data, flag_index, det_flags,
+    cudaError_t e = launch_offset_project(lease.wl, v, amp_offset, amplitudes, data_index, det_data, flag_index, det_flags,
                                           det_flag_mask, n_det, n_samp, (cudaStream_t)stream);
     if (e != cudaSuccess) return cuda_fail(e, "template_offset_project_signal launch");
     return ok();

@@ -493,6 +493,163 @@ __device__ __forceinline__ int loc2key32(const HealpixGeom& g, double dz, double
     }
 }
 
+// ----------------------------------------------------------------------------- compact run keys
+// The fused kernels (nside <= 4096) aggregate runs of equal pixels along each detector's
+// samples and only need a per-sample KEY that is equal for equal pixels; the pixel number itself
+// is formed once per run, when the run's sum is flushed (ckey_to_pix).  So the per-sample work
+// in the equatorial belt stops at the two floors:
+//   belt: key = (jp << 15) | jm            (jp, jm < 6.9 nside < 2^15)
+//   caps: key = 1 << 30 | payload          NEST: south << 26 | face << 24 | jp << 12 | jm
+//                                          RING: south << 26 | (north pixel, or npix - 1 - pixel)
+// Any two different pixels get different keys; one pixel can get two keys (the unwrapped
+// longitude of the incremental chain, OFF below, reaches a pixel from tt and tt + 4), which
+// only splits a run.  Keys are non-negative; -1 means "no pixel".
+constexpr int kCapBit = 1 << 30;
+
+// Floors of the HEALPix belt / caps with the longitude tt in quarter turns (OFF: tt + 1, unwrapped,
+// in (0.18, 5.82), see the fused kernel's incremental longitude).  The belt floors use one FMA
+// each: jp = floor(fma(-z, 0.75 N, N (tt + 1/2))), which differs from the rounding order of the
+// textbook expression (reading S6) only when the argument lies within ~2 ulp of an integer, i.e.
+// for directions within ~1e-15 rad of a pixel boundary (rule T1 allows 1e-12 rad).
+struct KeyConsts {
+    double dn, dn_half_m, dn_3q;  // N, N/2 - 1/2, 3N/4 (exact)
+};
+inline KeyConsts make_key_consts(int64_t nside) {
+    KeyConsts k;
+    k.dn = (double)nside;
+    k.dn_half_m = 0.5 * (double)nside - 0.5;
+    k.dn_3q = 0.75 * (double)nside;
+    return k;
+}
+
+// floor(x + 1/2) - ... : the belt floors as ROUND-TO-NEAREST of (argument - 1/2) on the fp64 pipe:
+// adding 1.5 2^52 rounds to an integer held in the low word (two fp64 adds of latency instead of
+// the ~34-cycle F2I.F64, measured on B200: scripts/fp64_microbench.cu).  It equals floor(argument)
+// except when the argument is within an ulp or so of an integer (ties, and the one rounding of the
+// shifted argument), i.e. for directions within ~1e-15 rad of a pixel boundary (rule T1).
+__device__ __forceinline__ int round_shifted(double x_minus_half) {
+    return __double2loint(x_minus_half + 6755399441055744.0);
+}
+
+template <bool NEST, bool OFF>
+__device__ __forceinline__ int loc2ckey(const HealpixGeom& g, const KeyConsts& kc, double dz, double tt, double t1m,
+                                        double dx, double dy) {
+    const double za = fabs(dz);
+    // the belt key is formed unconditionally (straight-line, so the scheduler can overlap it with
+    // independent work); only the caps branch.
+    // t1m = N (tt + 1/2) - 1/2;  jp = floor(N (tt + 1/2) - 3N/4 z), jm = floor(... + 3N/4 z)
+    const int bjp = round_shifted(fma(-dz, kc.dn_3q, t1m));
+    const int bjm = round_shifted(fma(dz, kc.dn_3q, t1m));
+    const int belt = (bjp << 15) | bjm;
+    if (za <= TB_TWO_THIRD) return belt;
+    const int nside = (int)g.nside;
+    const int m = nside - 1;
+    double tmp;
+    if (za < TB_CAP_SINTHETA_Z) {
+        tmp = __dmul_rn(g.dnside, fast_sqrt(__dmul_rn(3.0, __dsub_rn(1.0, za))));
+    } else {
+        const double sth = __dsqrt_rn(__dadd_rn(__dmul_rn(dx, dx), __dmul_rn(dy, dy)));
+        tmp = __ddiv_rn(__dmul_rn(g.dnside, sth), __dsqrt_rn(__ddiv_rn(__dadd_rn(1.0, za), 3.0)));
+    }
+    const int south = dz < 0.0 ? 1 : 0;
+    if (!NEST) {
+        const double tp = __dsub_rn(tt, small_int_to_double(floor_nonneg(tt)));
+        const int jp = floor_nonneg(__dmul_rn(tp, tmp));
+        const int jm = floor_nonneg(__dmul_rn(__dsub_rn(1.0, tp), tmp));
+        const int ir = jp + jm + 1;
+        int ip = floor_nonneg(__dmul_rn(tt, small_int_to_double(ir)));
+        if (OFF) {
+            ip -= ir;  // in [-0.82 ir, 4.82 ir)
+            if (ip < 0) ip += 4 * ir;
+        }
+        if (ip >= 4 * ir) ip -= 4 * ir;
+        // north: 2 ir (ir - 1) + ip; south: npix - 2 ir (ir + 1) + ip, stored as npix - 1 - pixel
+        const int p = south ? 2 * ir * (ir + 1) - 1 - ip : 2 * ir * (ir - 1) + ip;
+        return kCapBit | (south << 26) | p;
+    } else {
+        int ntt = floor_nonneg(tt);
+        if (!OFF && ntt > 3) ntt = 3;
+        const double tp = __dsub_rn(tt, small_int_to_double(ntt));
+        const int face = OFF ? ((ntt + 3) & 3) : ntt;
+        int jp = floor_nonneg(__dmul_rn(tp, tmp));
+        int jm = floor_nonneg(__dmul_rn(__dsub_rn(1.0, tp), tmp));
+        jp = min(jp, m);
+        jm = min(jm, m);
+        return kCapBit | (south << 26) | (face << 24) | (jp << 12) | jm;
+    }
+}
+
+// Pixel of a compact key (run flush; see loc2ckey).
+template <bool NEST, bool OFF>
+__device__ __forceinline__ int ckey_to_pix(int key, const HealpixGeom& g) {
+    const int nside = (int)g.nside;
+    const int m = nside - 1;
+    if (key & kCapBit) {
+        const int south = (key >> 26) & 1;
+        if (!NEST) {
+            const int p = key & ((1 << 26) - 1);
+            return south ? (int)g.npix - 1 - p : p;
+        }
+        const int face = ((key >> 24) & 3) + 8 * south;
+        const int jp = (key >> 12) & 0xfff, jm = key & 0xfff;
+        const int ix = south ? jp : m - jm;
+        const int iy = south ? jm : m - jp;
+        return face * (nside * nside) + (int)interleave16((uint32_t)ix, (uint32_t)iy);
+    }
+    const int jp = key >> 15, jm = key & 0x7fff;
+    if (!NEST) {
+        const int nl4 = 4 * nside;
+        const int ir = nside + 1 + jp - jm;
+        const int kshift = 1 - (ir & 1);
+        const int t1 = jp + jm - (OFF ? 3 : 1) * nside + kshift + 1 + 2 * nl4;
+        const int ip = (t1 >> 1) & (nl4 - 1);
+        return (int)g.ncap + nl4 * (ir - 1) + ip;
+    }
+    const int ifp = jp >> g.order;
+    const int ifm = jm >> g.order;
+    const int fmin = (ifp < ifm ? ifp : ifm) + (OFF ? 3 : 0);
+    const int face = (fmin & 3) + 4 * (1 + ifp - ifm);
+    const int ix = jm & m;
+    const int iy = (jp & m) ^ m;
+    return face * (nside * nside) + (int)interleave16((uint32_t)ix, (uint32_t)iy);
+}
+
+// The same as ckey_to_pix without branches (the run flush decodes 32 keys at once, belt and cap
+// keys mixed in one warp): both decodings are formed and one is selected.
+template <bool NEST, bool OFF>
+__device__ __forceinline__ int ckey_to_pix_bf(int key, const HealpixGeom& g) {
+    const int nside = (int)g.nside;
+    const int m = nside - 1;
+    const bool cap = key & kCapBit;
+    const int south = (key >> 26) & 1;
+    if (!NEST) {
+        const int nl4 = 4 * nside;
+        const int jp = key >> 15, jm = key & 0x7fff;
+        const int ir = nside + 1 + jp - jm;
+        const int kshift = 1 - (ir & 1);
+        const int t1 = jp + jm - (OFF ? 3 : 1) * nside + kshift + 1 + 2 * nl4;
+        const int belt = (int)g.ncap + nl4 * (ir - 1) + ((t1 >> 1) & (nl4 - 1));
+        const int p = key & ((1 << 26) - 1);
+        const int capp = south ? (int)g.npix - 1 - p : p;
+        return cap ? capp : belt;
+    }
+    // belt
+    const int bjp = (key >> 15) & 0x7fff, bjm = key & 0x7fff;
+    const int ifp = bjp >> g.order, ifm = bjm >> g.order;
+    const int fmin = (ifp < ifm ? ifp : ifm) + (OFF ? 3 : 0);
+    const int bface = (fmin & 3) + 4 * (1 + ifp - ifm);
+    const int bix = bjm & m, biy = (bjp & m) ^ m;
+    // cap
+    const int cjp = (key >> 12) & 0xfff, cjm = key & 0xfff;
+    const int cface = ((key >> 24) & 3) + 8 * south;
+    const int cix = south ? cjp : m - cjm;
+    const int ciy = south ? cjm : m - cjp;
+    const int face = cap ? cface : bface;
+    const int ix = cap ? cix : bix;
+    const int iy = cap ? ciy : biy;
+    return face * (nside * nside) + (int)interleave16((uint32_t)ix, (uint32_t)iy);
+}
+
 // Pixel of a run key (see loc2key32).
 template <bool NEST>
 __device__ __forceinline__ int key_to_pix32(int key, const HealpixGeom& g) {

@@ -7,7 +7,7 @@
 //     item, fetched one item ahead) in chunk-major order, so the warps in flight cover a short
 //     time window of the focal plane and the sky footprint they scatter into stays L2-resident.
 //   * Each lane holds its detector's frame in registers for the whole item:
-//       u = R(f) z, v = R(f) x, w = R(f) y, det_scale*cal, det_scale*eta*cal.
+//       u = R(f) z, v = R(f) x, w = R(f) y and its noise-weight scales.
 //   * An item is a STREAM OF BLOCKS of kBlk = 16 samples through two warp-private shared
 //     buffers: while block i is computed, lane 0's bulk tensor copies (TMA, mbarrier-completed;
 //     per-lane cp.async when the TMA constraints fail) stage block i+1 — the TOD tile [32 x 16]
@@ -15,20 +15,28 @@
 //     flags.  Lanes 0..15 turn them into the per-sample state (boresight rotation matrix B —
 //     identity if shared-flagged, reading S2), lanes 16..31 into cos/sin 4 chi; every lane then
 //     walks the 16 samples reading that state as shared-memory broadcasts.  Boresight, HWP and
-//     shared flags are read from HBM once per 32 detectors.
+//     shared flags are read from HBM once per 32 detectors.  (Measured and rejected: a 7 KB
+//     single-buffer staging with two TOD half tiles for 24 warps/SM — the 80-register bound
+//     added 35 % instructions and the half-block lookahead exposed TMA latency: C2 0.56 ms vs
+//     0.47 ms.)
 //   * Per det-sample: dir = B u, bx = (B v)_z, by = -(B w)_z, the longitude carried
 //     incrementally along the lane's samples (one reciprocal shared with the weights), the
-//     HEALPix run key, cos/sin 2psi algebraically, the HWP angle addition.
+//     compact HEALPix run key (belt: the two floors only, device_math.cuh loc2ckey), cos/sin 2psi
+//     algebraically, the HWP angle addition.
 //   * Map accumulation is RUN-LENGTH aggregated per lane along time: consecutive samples of one
-//     detector in the same pixel are summed in registers and flushed with one fp64 `red` per
-//     Stokes component when the pixel changes; hit-submap flags are gathered per CTA in shared
-//     memory.  SCAN mode gathers the map instead (cached per lane across the run) and updates
-//     the staged TOD tile, written back after each block.
+//     detector with the same key are summed in registers; when the key changes the lane
+//     flushes its run: key -> pixel, submap, global2local and hit flag from a per-CTA
+//     shared-memory cache, one fp64 `red` per Stokes component (measured against a converged
+//     per-warp flush queue: the queue won 2 % at C2 and lost 8-10 % at C3/C5, where some lane of
+//     the 32 changes pixel at most samples anyway).
+//   * SCAN mode gathers the map instead (cached per lane across the run) and updates the
+//     staged TOD, written back after each half block.
 #include <cuda.h>  // CUtensorMap (the encoder is fetched through the runtime; no -lcuda)
 #include <cuda_runtime.h>
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 
@@ -42,106 +50,34 @@ namespace {
 #ifndef TB_FUSED_MINB
 #define TB_FUSED_MINB 2  // resident CTAs per SM the register allocation is bounded for
 #endif
-#ifndef TB_FUSED_DPL_MAX
-#define TB_FUSED_DPL_MAX 1  // detectors per lane (2 when n_det > 32 and DPL_MAX = 2)
-#endif
-#ifndef TB_WARPS
-#define TB_WARPS 8
-#endif
-constexpr int kWarps = TB_WARPS;  // warps per CTA
-#ifndef TB_BLK
-#define TB_BLK 16
-#endif
-constexpr int kBlk = TB_BLK;  // samples per block (8 or 16)
-constexpr int kRowStep = 32 / kBlk;  // TOD rows staged per cp.async instruction
-#ifndef TB_KUNROLL
-#define TB_KUNROLL 1
-#endif
-constexpr int kKUnroll = TB_KUNROLL;  // unroll of the per-sample loop
-#ifndef TB_INCR
-#define TB_INCR 1  // incremental longitude along each detector's samples (see stage_a)
-#endif
-#ifndef TB_FOLD
-#define TB_FOLD 1  // det_scale (and eta cal) applied once per run at the flush, not per det-sample
-#endif
-#ifndef TB_TTOFF
-#define TB_TTOFF 1  // 32-bit keys: longitude carried as tt + 1 without wrapping (see stage_a)
-#endif
-#ifndef TB_INCR_BF
-#define TB_INCR_BF 1  // branch-free incremental-longitude series (see stage_a; measured -0.5..1 % C2)
-#endif
-#ifndef TB_DEFER
-#define TB_DEFER 1  // a det-sample's contribution is folded into its run one sample later
-#endif
-#ifndef TB_HITDEDUP
-#define TB_HITDEDUP 0  // shared hit flags: compare with the lane's last submap first (measured: +1 % C2, +2 % C3)
-#endif
-constexpr int kPad = kBlk + 1;
+constexpr int kWarps = 8;  // warps per CTA
+constexpr int kBlk = 16;   // samples per block
+constexpr unsigned kFull = 0xffffffffu;
 
-// per-sample state: B[0..8], c4, s4, mode (as a double: 1 pixelise, 2 shared-flagged)
-struct SampleState {
-    double v[12];
-};
+__device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
 
-// Raw inputs of one block (filled by cp.async).
-template <int DPL>
-struct alignas(16) RawBlock {
-    double tod[32 * DPL][kPad];
-    double bore[kBlk][4];
-    double hwp[kBlk];
-    uint8_t flg[32 * DPL][kBlk + 4];  // 5 aligned words covering each row's 16 flag bytes
-    uint8_t sflg[kBlk + 8];           // 5 aligned words covering the 16 shared flags
-};
-
-template <int DPL>
-struct WarpSmem {
-    RawBlock<DPL> buf[2];
-    SampleState st[kBlk];
-};
-
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
-    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
+__device__ __forceinline__ void cp_async8(unsigned dst, const void* gmem) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(dst), "l"(gmem) : "memory");
 }
-// L2 evict-first policy for the streamed-once inputs (TOD, det flags): they must not push
-// the map lines being accumulated out of L2 (the map's red operations miss otherwise).
+__device__ __forceinline__ void cp_async8_pol(unsigned dst, const void* gmem, uint64_t pol) {
+    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 8, %2;\n" ::"r"(dst), "l"(gmem), "l"(pol)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
+
+// L2 evict-first policy for the streamed-once inputs (TOD, det flags): they must not push the
+// map lines being accumulated out of L2.
 __device__ __forceinline__ uint64_t evict_first_policy() {
     uint64_t pol;
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;\n" : "=l"(pol));
     return pol;
 }
-__device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
-    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async8_stream(void* smem, const void* gmem, uint64_t pol) {
-    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
-    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 8, %2;\n" ::"r"(s), "l"(gmem), "l"(pol)
-                 : "memory");
-}
-__device__ __forceinline__ void cp_async4(void* smem, const void* gmem) {
-    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(s), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
 
-// Copy the aligned 4-byte words covering bytes [p, p + n) (n <= 16) to dst[0..20); the
-// caller reads byte i of the range at dst[(p & 3) + i].  Words past the range are skipped,
-// so nothing beyond the aligned word holding the last byte is read.
-__device__ __forceinline__ void cp_async_bytes(uint8_t* dst, const uint8_t* p, int n, int w) {
-    const uint8_t* w0 = reinterpret_cast<const uint8_t*>(reinterpret_cast<uintptr_t>(p) & ~uintptr_t(3));
-    if (w0 + 4 * w < p + n) cp_async4(dst + 4 * w, w0 + 4 * w);
-}
-
-// ----------------------------------------------------------------------------- TMA path
-// When the inputs satisfy the tensor-memory-accelerator constraints (n_samp % 16 == 0 and
-// 16-byte aligned arrays), lane 0 moves a whole block with five
-// bulk tensor copies that complete on a per-buffer mbarrier, instead of 32 lanes issuing
-// ~30 cp.async each with 64-bit address arithmetic.  The TOD tile [32 det][16 samples] lands
-// 128-byte-swizzled (row r's 16-byte chunk c at c ^ (r & 7)), so the per-sample column read
-// tod[lane][k] is a 4-wavefront access without padding bytes.  Boxes start at multiples of 16
-// samples (a box must start 16-byte aligned in every staged row).
+// ----------------------------------------------------------------------------- TMA
 struct alignas(64) TmaMaps {
     CUtensorMap tod;   // f64 [n_det][n_samp], box {16, 32}, SWIZZLE_128B
     CUtensorMap flg;   // u8  [n_det][n_samp], box {16, 32}
@@ -149,25 +85,6 @@ struct alignas(64) TmaMaps {
     CUtensorMap hwp;   // f64 [n_samp],        box {16}
     CUtensorMap sflg;  // u8  [n_samp],        box {16}
 };
-
-// Every TMA destination is 128-byte aligned; the 16 shared-flag bytes of a buffer share their
-// 128-byte slot with that buffer's mbarrier, so a warp's staging area is exactly 12 KB.
-struct alignas(128) SflgSlot {
-    uint8_t f[16];
-    unsigned long long mbar;
-    uint8_t pad[104];
-};
-struct alignas(1024) TmaWarpSmem {
-    double tod[2][32][16];           // 1024-aligned (the 128-byte swizzle pattern spans 1 KB)
-    uint8_t flg[2][32][16];
-    double bore[2][16][4];
-    double hwp[2][16];
-    SflgSlot sf[2];
-    double st[16][12];               // SampleState[kBlk]
-};
-static_assert(sizeof(TmaWarpSmem) == 12288, "TMA staging area: 12 KB per warp");
-
-__device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
 
 __device__ __forceinline__ void mbar_init(unsigned long long* bar) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(smem_u32(bar)) : "memory");
@@ -200,7 +117,6 @@ __device__ __forceinline__ void tma_2d(void* dst, const CUtensorMap* m, int c0, 
         "l"(m), "r"(c0), "r"(c1), "r"(smem_u32(bar))
         : "memory");
 }
-// streamed-once TOD / det flags with an L2 evict-first hint (see evict_first_policy)
 __device__ __forceinline__ void tma_2d_stream(void* dst, const CUtensorMap* m, int c0, int c1,
                                               unsigned long long* bar, uint64_t pol) {
     asm volatile(
@@ -210,7 +126,33 @@ __device__ __forceinline__ void tma_2d_stream(void* dst, const CUtensorMap* m, i
         : "memory");
 }
 
-// Pixel index type: 32-bit up to nside 8192 (12 nside^2 < 2^31), else 64-bit.
+// fp64 / fp32 map reductions (no return value: RED, executed in L2)
+__device__ __forceinline__ void red_f64(double* p, double v) {
+    asm volatile("red.global.add.f64 [%0], %1;" ::"l"(p), "d"(v) : "memory");
+}
+__device__ __forceinline__ void red_f32(float* p, float v) {
+    asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
+}
+
+// Per-warp shared memory: two staging buffers and the per-sample state (12 KB).  Every TMA
+// destination is 128-byte aligned; the 16 shared-flag bytes of a buffer share their 128-byte slot
+// with that buffer's mbarrier.
+struct alignas(128) SflgSlot {
+    uint8_t f[16];
+    unsigned long long mbar;
+    uint8_t pad[104];
+};
+struct alignas(1024) WarpSmem {
+    double tod[2][32][16];  // 1024-aligned (the 128-byte swizzle pattern spans 1 KB)
+    uint8_t flg[2][32][16];
+    double bore[2][16][4];
+    double hwp[2][16];
+    SflgSlot sf[2];
+    double st[16][12];      // per-sample state: B[0..8], c4, 2 s4, s4 / 2
+};
+static_assert(sizeof(WarpSmem) == 12288, "12 KB per warp");
+
+// Pixel index / key type: 32-bit compact keys up to nside 4096, else the 64-bit pixel itself.
 template <bool WIDE>
 struct PixT;
 template <>
@@ -222,137 +164,155 @@ struct PixT<true> {
     using T = int64_t;
 };
 
-// Submap of a pixel (shift when n_pix_submap is a power of two).
-template <typename P>
-__device__ __forceinline__ int64_t submap_of(P pix, const MapGeom& mg) {
-    return mg.sm_shift >= 0 ? (int64_t)(pix >> mg.sm_shift) : (int64_t)pix / mg.n_pix_submap;
+// Per-CTA shared state besides the warps' areas: the global2local cache (int16: local submap,
+// 0x7fff = no storage, bit 15 = hit) and whether it is in use.
+struct CtaMem {
+    uint16_t* g2l;  // [n_submap] when cached
+    bool cached;
+};
+constexpr uint16_t kNoLoc = 0x7fff;
+constexpr uint16_t kHitBit = 0x8000;
+
+// Map geometry and the key -> (local submap, pixel in submap) step of a run flush.
+template <bool NEST, bool OFF, bool WIDE>
+__device__ __forceinline__ int64_t key_to_pixel(typename PixT<WIDE>::T key, const HealpixGeom& g) {
+    if constexpr (WIDE)
+        return key;
+    else
+        return ckey_to_pix<NEST, OFF>(key, g);
 }
 
-// Pixel of a run key: 32-bit NEST keys are the cheap (face, iy, ix) packing of loc2key32;
-// 64-bit keys (nside > 8192) and RING keys are the pixel itself.
-template <bool NEST, bool WIDE>
-__device__ __forceinline__ typename PixT<WIDE>::T key_to_pix(typename PixT<WIDE>::T key, const HealpixGeom& g) {
-    if constexpr (WIDE) {
-        return key;
+// Resolve the storage of a pixel's submap and mark the submap hit.  Returns the map element
+// offset (in elements of nnz) or -1 if the submap has no storage.
+__device__ __forceinline__ int64_t locate(int64_t pix, const FusedArgs& a, const CtaMem& cm) {
+    const MapGeom& mg = a.map;
+    int64_t sm, lp;
+    if (mg.sm_shift >= 0) {
+        sm = pix >> mg.sm_shift;
+        lp = pix & (mg.n_pix_submap - 1);
     } else {
-        return key_to_pix32<NEST>(key, g);
+        sm = pix / mg.n_pix_submap;
+        lp = pix - sm * mg.n_pix_submap;
+    }
+    int64_t loc;
+    if (cm.cached) {
+        const uint16_t v = cm.g2l[sm];
+        if (a.hit_submaps) cm.g2l[sm] = v | kHitBit;  // idempotent: every writer stores the same value
+        const unsigned l = v & 0x7fffu;
+        loc = l == kNoLoc ? -1 : (int64_t)l;
+    } else {
+        if (a.hit_submaps) a.hit_submaps[sm] = 1;
+        loc = __ldg(&mg.global2local[sm]);
+    }
+    return loc < 0 ? -1 : loc * mg.n_pix_submap + lp;
+}
+
+// Reading R3: (r1, r2) <- diag(1, +-1) R(-4 gamma_det) (r1, r2).  Out of line: the full-range
+// sincos is large and this variant path must not grow the hot loop's code.
+__device__ __noinline__ double2 gamma_rotate(double r1, double r2, const double* gamma, int iau, int64_t det) {
+    double s4, c4;
+    sincos(4.0 * __ldg(&gamma[det]), &s4, &c4);
+    const double q = fma(c4, r1, s4 * r2);
+    const double u = fma(c4, r2, -s4 * r1);
+    return make_double2(q, iau ? -u : u);
+}
+
+// One run's contribution into the map (prescaled sums; reading R3's rotation by -4 gamma and
+// the IAU sign of U applied here when a gamma array is given).
+template <int NNZ>
+__device__ __forceinline__ void add_run(int64_t elem, double r0, double r1, double r2, const FusedArgs& a,
+                                        int64_t det) {
+    if (elem < 0) return;
+    if (NNZ == 3 && a.gamma != nullptr && a.hwp != nullptr) {
+        const double2 v = gamma_rotate(r1, r2, a.gamma, a.iau, det);
+        r1 = v.x;
+        r2 = v.y;
+    }
+    if (a.map_f32) {
+        float* dst = reinterpret_cast<float*>(a.zmap) + elem * NNZ;
+        red_f32(dst, (float)r0);
+        if (NNZ == 3) {
+            red_f32(dst + 1, (float)r1);
+            red_f32(dst + 2, (float)r2);
+        }
+    } else {
+        double* dst = a.zmap + elem * NNZ;
+        red_f64(dst, r0);
+        if (NNZ == 3) {
+            red_f64(dst + 1, r1);
+            red_f64(dst + 2, r2);
+        }
     }
 }
 
+// The general run flush (64-bit keys, non-power-of-two submaps, uncached global2local, fp32
+// maps, the reading-R3 rotation), out of line so that the hot loop's code stays small.
+template <bool NEST, int NNZ, bool OFF, bool WIDE>
+__device__ __noinline__ void drain_general(typename PixT<WIDE>::T key, double r0, double r1, double r2, double* zmap,
+                                           int map_f32, uint8_t* hit_submaps, const int64_t* global2local,
+                                           int sm_shift, int64_t n_pix_submap, uint16_t* g2l_cache, bool cached,
+                                           const double* gamma, bool have_hwp, int iau, int64_t det, HealpixGeom g) {
+    const int64_t pix = key_to_pixel<NEST, OFF, WIDE>(key, g);
+    int64_t sm, lp;
+    if (sm_shift >= 0) {
+        sm = pix >> sm_shift;
+        lp = pix & (n_pix_submap - 1);
+    } else {
+        sm = pix / n_pix_submap;
+        lp = pix - sm * n_pix_submap;
+    }
+    int64_t loc;
+    if (cached) {
+        const uint16_t v = g2l_cache[sm];
+        if (hit_submaps) g2l_cache[sm] = v | kHitBit;
+        const unsigned l = v & 0x7fffu;
+        loc = l == kNoLoc ? -1 : (int64_t)l;
+    } else {
+        if (hit_submaps) hit_submaps[sm] = 1;
+        loc = __ldg(&global2local[sm]);
+    }
+    if (loc < 0) return;
+    const int64_t elem = loc * n_pix_submap + lp;
+    if (NNZ == 3 && gamma != nullptr && have_hwp) {
+        double s4, c4;
+        sincos(4.0 * __ldg(&gamma[det]), &s4, &c4);
+        const double q = fma(c4, r1, s4 * r2);
+        const double u = fma(c4, r2, -s4 * r1);
+        r1 = q;
+        r2 = iau ? -u : u;
+    }
+    if (map_f32) {
+        float* dst = reinterpret_cast<float*>(zmap) + elem * NNZ;
+        red_f32(dst, (float)r0);
+        if (NNZ == 3) {
+            red_f32(dst + 1, (float)r1);
+            red_f32(dst + 2, (float)r2);
+        }
+    } else {
+        double* dst = zmap + elem * NNZ;
+        red_f64(dst, r0);
+        if (NNZ == 3) {
+            red_f64(dst + 1, r1);
+            red_f64(dst + 2, r2);
+        }
+    }
+}
+
+// Per-lane state of an item.
 template <typename P>
 struct Slot {
     double u0, u1, u2, v0, v1, v2, w0, w1, w2;
-    double s_cal;   // det_scale * cal       (I weight folded into the noise weight)
-    double s_eta;   // det_scale * eta * cal (Q/U amplitude folded into the noise weight)
-    double etacal;  // debug outputs only
-    P run_key;            // key of the run being aggregated (-1: none)
-    P run_lp;             // its pixel's index inside the submap
-    int64_t run_loc;      // global2local of the run's submap, LOADED WHEN THE RUN STARTS
-    P last_sm;            // last submap this lane marked in hit_submaps (generic path)
-    int64_t last_loc;     // SCAN: global2local of last_sm
-    double r0, r1, r2;
-    P pend_key;           // pending (not yet aggregated) det-sample
-    double p0, p1, p2;
-    double px, py, ptt;   // INCR mode: projected direction and tt of the lane's previous sample
+    double sI;      // det_scale * cal             (I)
+    double sQ, sU;  // det_scale * eta * cal, times 2 for U (the run sums carry bx by, not 2 bx by) and
+                    // the IAU sign when no gamma rotation follows in add_run
+    double etacal;  // debug outputs / SCAN
+    double r0, r1, r2;  // run sums: sum tod, sum tod cq / r, sum tod sq' / r
+    double px, py, ptt; // incremental longitude: projected direction and tt of the previous sample
+    P run_key;          // key of the run being aggregated (-1: none)
+    int64_t run_elem;   // SCAN: map element of the cached run (-1: none)
+    int64_t det;
     bool ok;
 };
-
-// Per-CTA shared memory besides the warps' staging areas: the bit-spread table of the NEST
-// interleave (spread[b] = the 8 bits of b moved to the even bit positions) and the CTA's
-// hit-submap flags (MapGeom::shared_hits).
-struct CtaMem {
-    const uint16_t* spread;  // [256]
-    uint8_t* hits;           // [n_submap] when MapGeom::shared_hits
-};
-constexpr int kSpreadBytes = 512;
-
-// Pixel of a 32-bit run key with the bit interleave from the shared spread table: 2 (nside <=
-// 256) or 4 table loads instead of the ~16 instructions of interleave16 — this runs at every run
-// start, and with 32 detectors per warp some lane starts a run at most samples.
-template <bool NEST>
-__device__ __forceinline__ int key_to_pix_tab(int key, const HealpixGeom& g, const uint16_t* spread) {
-    if (!NEST) return key;
-    const int m = (int)g.nside - 1;
-    const uint32_t ix = (uint32_t)(key & m), iy = (uint32_t)((key >> g.order) & m);
-    uint32_t v = spread[ix & 255u] | ((uint32_t)spread[iy & 255u] << 1);
-    if (g.order > 8) v |= (spread[ix >> 8] | ((uint32_t)spread[iy >> 8] << 1)) << 16;
-    return (key & ~((1 << (2 * g.order)) - 1)) | (int)v;
-}
-
-// A run starts: mark its submap hit (as A2 does) and issue the global2local lookup now, so
-// the load latency is hidden behind the run's samples instead of stalling the flush.  The hit
-// flag is stored only when the lane's submap CHANGES: thousands of warps re-writing the same
-// few bytes of hit_submaps serialise in L2 and cost as much as the whole computation.
-// Sets sl.run_loc (-1: the submap has no storage) and sl.run_lp.
-template <bool NEST, bool WIDE>
-__device__ __forceinline__ void start_run(typename PixT<WIDE>::T key, const FusedArgs& a, const HealpixGeom& g,
-                                          Slot<typename PixT<WIDE>::T>& sl, const CtaMem& cm) {
-    using P = typename PixT<WIDE>::T;
-    const MapGeom& mg = a.map;
-    P pix;
-    if constexpr (WIDE)
-        pix = key;
-    else
-        pix = key_to_pix_tab<NEST>(key, g, cm.spread);
-    P sm;
-    if (mg.sm_shift >= 0) {
-        sm = pix >> mg.sm_shift;
-        sl.run_lp = pix & (P)(mg.n_pix_submap - 1);
-    } else {
-        sm = pix / (P)mg.n_pix_submap;
-        sl.run_lp = pix - sm * (P)mg.n_pix_submap;
-    }
-#ifndef TB_X_NOHIT
-    if (mg.shared_hits) {
-        // the CTA's shared copy (idempotent store, no atomic; see the kernel end)
-#if TB_HITDEDUP
-        if (sm != sl.last_sm) {
-            cm.hits[sm] = 1;
-            sl.last_sm = sm;
-        }
-#else
-        cm.hits[sm] = 1;
-#endif
-    } else if (a.hit_submaps && sm != sl.last_sm) {
-        a.hit_submaps[sm] = 1;
-        sl.last_sm = sm;
-    }
-#endif
-#ifdef TB_X_NOG2L
-    sl.run_loc = sm;
-#else
-    sl.run_loc = __ldg(&mg.global2local[sm]);
-#endif
-}
-
-// A run ends: one fp64 red per Stokes component (nothing if the submap has no storage).  Up to
-// nside 8192 the map element index fits 32 bits (< 12 * 8192^2 pixels), so the address is one
-// IMAD + one IMAD.WIDE.U32.  With TB_FOLD the run sums are unscaled (sum of tod, of tod w/r)
-// and det_scale * cal, det_scale * eta * cal are applied here, once per run.
-template <int NNZ, bool WIDE>
-__device__ __forceinline__ void flush(const Slot<typename PixT<WIDE>::T>& sl, const FusedArgs& a) {
-    if (sl.run_loc < 0) return;
-    double* dst;
-    if constexpr (WIDE) {
-        dst = a.zmap + (sl.run_loc * a.map.n_pix_submap + sl.run_lp) * NNZ;
-    } else {
-        const unsigned idx = (unsigned)sl.run_loc * (unsigned)a.map.n_pix_submap + (unsigned)sl.run_lp;
-        dst = a.zmap + (size_t)idx * NNZ;
-    }
-#if TB_FOLD
-    atomicAdd(dst, sl.r0 * sl.s_cal);
-    if (NNZ == 3) {
-        atomicAdd(dst + 1, sl.r1 * sl.s_eta);
-        atomicAdd(dst + 2, sl.r2 * sl.s_eta);
-    }
-#else
-    atomicAdd(dst, sl.r0);
-    if (NNZ == 3) {
-        atomicAdd(dst + 1, sl.r1);
-        atomicAdd(dst + 2, sl.r2);
-    }
-#endif
-}
 
 template <typename P>
 __device__ __forceinline__ void load_slot(Slot<P>& sl, const FusedArgs& a, int64_t d, bool ok, int64_t dfallback) {
@@ -367,26 +327,26 @@ __device__ __forceinline__ void load_slot(Slot<P>& sl, const FusedArgs& a, int64
     const double eps = __ldg(&a.epsilon[dd]);
     const double scale = __ldg(&a.det_scale[dd]);
     sl.etacal = (1.0 - eps) / (1.0 + eps) * a.cal;
-    // a lane without a detector contributes exactly 0 (aggregate() adds unconditionally)
-    sl.s_cal = ok ? scale * a.cal : 0.0;
-    sl.s_eta = ok ? scale * sl.etacal : 0.0;
+    const bool rot = a.gamma != nullptr && a.hwp != nullptr;
+    const double usign = (a.iau && !rot) ? -1.0 : 1.0;
+    // a lane without a detector contributes exactly 0
+    sl.sI = ok ? scale * a.cal : 0.0;
+    sl.sQ = ok ? scale * sl.etacal : 0.0;
+    sl.sU = 2.0 * usign * sl.sQ;
     sl.run_key = -1;
-    sl.run_lp = 0;
-    sl.run_loc = -1;
-    sl.last_sm = -1;
-    sl.last_loc = -1;
+    sl.run_elem = -1;
     sl.r0 = sl.r1 = sl.r2 = 0.0;
-    sl.pend_key = -1;
-    sl.p0 = sl.p1 = sl.p2 = 0.0;
     sl.px = sl.py = sl.ptt = 0.0;  // dot = 0: the item's first sample takes the full arctangent
+    sl.det = dd;
     sl.ok = ok;
 }
 
 // The straight-line fp64 part of one det-sample (A1 -> direction, A3 weights and the A2
-// longitude): no branches, so two of them can be interleaved by the scheduler (pair loop).
+// longitude).
 struct StageA {
     double dx, dy, dz, tt;
-    double cw, sw, invr;  // r cos 2(psi + 2 chi), r sin 2(psi + 2 chi), 1/r
+    double cw, sw, invr;  // r cos 2(psi + 2 chi), r sin 2(psi + 2 chi) / 2, 1/r
+    double t1m;           // N (tt + 1/2) - 1/2: the belt floors' common term (see loc2ckey_t1m)
 };
 
 // (2/pi) atan(t) = t Q(t^2) for |t| <= kIncrMax = 0.01 (TB_INCR_MAX, in the constant bank): the
@@ -394,9 +354,13 @@ struct StageA {
 __constant__ double kIncrQ[4] = {0.63661977236758134308, -0.21220659078919378103, 0.12732395447351626862,
                                  -0.090945681766797334729};
 
+// OFF: 32-bit keys with the incremental longitude carried as tt + 1 WITHOUT wrapping (see below).
+template <int NNZ, typename P>
+constexpr bool kOff = NNZ == 3 && sizeof(P) == 4;
+
 template <int NNZ, bool HWP, typename P>
-__device__ __forceinline__ StageA stage_a(Slot<P>& sl, const double* x) {
-    constexpr bool TTOFF = TB_TTOFF && TB_INCR && sizeof(P) == 4;
+__device__ __forceinline__ StageA stage_a(Slot<P>& sl, const double* x, const KeyConsts& kc) {
+    constexpr bool OFF = kOff<NNZ, P>;
     StageA o;
     o.dx = x[0] * sl.u0 + x[1] * sl.u1 + x[2] * sl.u2;
     o.dy = x[3] * sl.u0 + x[4] * sl.u1 + x[5] * sl.u2;
@@ -405,314 +369,213 @@ __device__ __forceinline__ StageA stage_a(Slot<P>& sl, const double* x) {
     if (NNZ == 3) {
         const double bx = x[6] * sl.v0 + x[7] * sl.v1 + x[8] * sl.v2;
         const double by = -(x[6] * sl.w0 + x[7] * sl.w1 + x[8] * sl.w2);
-#ifdef TB_X_NOATAN
-        o.tt = fabs(o.dx) * 3.9; o.cw = bx; o.sw = by; o.invr = 1.0;  // ablation: no longitude/weights arithmetic
-#elif TB_INCR
         // INCREMENTAL LONGITUDE: consecutive samples of a detector
         // are close on the sky, so tt(s) = tt(s') + (2/pi) atan(t) with t = tan(phi(s) - phi(s'))
         // = cross / dot of the projected directions of s and of this lane's previous processed
-        // sample s' — a 4-term series instead of the octant reduction, the 11-term polynomial and
-        // the octant bookkeeping.  Each step adds ~1 ulp of tt (~4e-16 quarter turns); the chain
-        // restarts from the full arctangent at every item (<= 128 samples), so the drift stays
-        // ~1e-15 rad, far inside rule T1's 1e-12 rad.  The ONE reciprocal 1/(dot r) still serves
-        // both t and the weights' 1/r.  Lanes whose step is large (|t| > 0.01: near a pole, after
-        // a gap) or that have no previous sample (dot = 0) take the full path.
+        // sample s' — a 4-term series instead of the octant reduction and the 11-term polynomial.
+        // Each step adds ~1 ulp of tt; the chain restarts from the full arctangent at every item
+        // (<= 128 samples), so the drift stays ~1e-15 rad, far inside rule T1's 1e-12 rad.  The
+        // ONE reciprocal 1/(dot r) serves both t and the weights' 1/r.  Lanes whose step is large
+        // (|t| > 0.01: near a pole, after a gap) or that have no previous sample (dot = 0) take
+        // the full path.  The series is evaluated for every sample (NaN at dot = 0, no traps on
+        // the GPU), so only the rare full path is a branch.
         const double bx2 = fma(bx, bx, TB_TINY);
         const double r = fma(by, by, bx2);
         o.cw = fma(-by, by, bx2);
-        o.sw = (bx + bx) * by;
+        o.sw = bx * by;  // half of r sin 2 psi: the factor 2 is folded into the U scale
         const double cross = fma(sl.px, o.dy, -(sl.py * o.dx));
         const double dot = fma(sl.px, o.dx, sl.py * o.dy);
+        const double cr = cross * r;  // off the reciprocal's critical path
         const double inv = fast_rcp(dot * r);
-        // |cross| < kIncrMax dot  <=>  dot > 0 and |t| < kIncrMax (t = cross / dot); false at
-        // dot = 0 (no previous sample) and for steps beyond a quarter turn; one DFMA + DSETP,
-        // resolved before the reciprocal's result is needed
-#if TB_INCR_BF
-        // branch-free common path: the series is evaluated for every sample (NaN at dot = 0, no
-        // traps on the GPU) and only the rare full-arctangent path is a branch, so the scheduler
-        // can interleave the series with the surrounding straight-line code
+        // the belt floors need N (tt + 1/2) - 1/2 = N t q + (N ptt + N/2 - 1/2): the second term is
+        // formed while the reciprocal is in flight, so the key path after t is short (Estrin
+        // form of q: depth 2 instead of 3)
+        const double pre = fma(kc.dn, sl.ptt, kc.dn_half_m);
         {
-            const double t = cross * (r * inv);
+            const double t = cr * inv;
             o.invr = dot * inv;
             const double s2 = t * t;
-            double q = fma(kIncrQ[3], s2, kIncrQ[2]);
-            q = fma(q, s2, kIncrQ[1]);
-            q = fma(q, s2, kIncrQ[0]);
+            const double nt = kc.dn * t;  // exact (power-of-two scale)
+            const double qa = fma(kIncrQ[1], s2, kIncrQ[0]);
+            const double qb = fma(kIncrQ[3], s2, kIncrQ[2]);
+            const double q = fma(s2 * s2, qb, qa);
             double tt = fma(t, q, sl.ptt);
-            if constexpr (!TTOFF) {
+            if constexpr (!OFF) {
                 if (__double2hiint(tt) < 0) tt += 4.0;
                 if (__double2hiint(tt) >= 0x40100000) tt -= 4.0;
             }
             o.tt = tt;
+            o.t1m = fma(nt, q, pre);
         }
+        // |cross| < kIncrMax dot  <=>  dot > 0 and |t| < kIncrMax; false at dot = 0 and for steps
+        // beyond a quarter turn
         if (!(fma(TB_INCR_MAX, dot, -fabs(cross)) > 0.0)) {
-#else
-        if (fma(TB_INCR_MAX, dot, -fabs(cross)) > 0.0) {
-            const double t = cross * (r * inv);
-            o.invr = dot * inv;
-            const double s2 = t * t;
-            double q = fma(kIncrQ[3], s2, kIncrQ[2]);
-            q = fma(q, s2, kIncrQ[1]);
-            q = fma(q, s2, kIncrQ[0]);
-            double tt = fma(t, q, sl.ptt);
-            if constexpr (!TTOFF) {
-                if (__double2hiint(tt) < 0) tt += 4.0;
-                if (__double2hiint(tt) >= 0x40100000) tt -= 4.0;
-            }
-            o.tt = tt;
-        } else {
-#endif
-            // TTOFF: the chain is carried as tt + 1 WITHOUT wrapping: it restarts here from a
-            // value in [1, 5) and drifts by at most 127 steps of (2/pi) atan(0.01) = 0.0064
-            // within an item, so it stays in (0.18, 5.82); loc2key32<NEST, true> folds it back
-            o.tt = lon_pol_raw(o.dx, o.dy, bx, by, o.cw, o.sw, o.invr) + (TTOFF ? 1.0 : 0.0);
+            // OFF: the chain is carried as tt + 1 WITHOUT wrapping: it restarts here from a value in
+            // [1, 5) and drifts by at most 127 steps of (2/pi) atan(0.01) = 0.0064 within an item,
+            // so it stays in (0.18, 5.82); loc2ckey<NEST, true> folds it back
+            double A, B;
+            o.tt = lon_pol_raw(o.dx, o.dy, bx, by, A, B, o.invr) + (OFF ? 1.0 : 0.0);
+            o.t1m = fma(kc.dn, o.tt, kc.dn_half_m);
         }
         sl.px = o.dx;
         sl.py = o.dy;
         sl.ptt = o.tt;
-#else
-        o.tt = lon_pol_raw(o.dx, o.dy, bx, by, o.cw, o.sw, o.invr);  // one shared reciprocal
-#endif
         if (HWP) {
-            const double c4 = x[9], s4 = x[10];
-            const double cq = o.cw * c4 - o.sw * s4;
-            const double sq = o.sw * c4 + o.cw * s4;
+            // (cq, sq') = rotation of (cw, 2 sw') by 4 chi, with sq' = sq / 2:
+            // x[9] = cos 4chi, x[10] = 2 sin 4chi, x[11] = sin 4chi / 2
+            const double cq = fma(-o.sw, x[10], o.cw * x[9]);
+            const double sq = fma(o.sw, x[9], o.cw * x[11]);
             o.cw = cq;
             o.sw = sq;
         }
     } else {
         o.tt = quarter_turns(o.dx, o.dy);
+        o.t1m = fma(kc.dn, o.tt, kc.dn_half_m);
     }
     return o;
 }
 
-// The HEALPix floors and integer part (branches: equatorial belt / caps): the run key.
+// The HEALPix key of a det-sample (-1: no pixel).
 template <bool NEST, int NNZ, bool WIDE>
-__device__ __forceinline__ typename PixT<WIDE>::T stage_b(const StageA& o, bool pixelise, bool ok,
-                                                         const HealpixGeom& g) {
+__device__ __forceinline__ typename PixT<WIDE>::T stage_b(const StageA& o, bool pixelise, const HealpixGeom& g,
+                                                         const KeyConsts& kc) {
     using P = typename PixT<WIDE>::T;
-    P key = -1;
-    if (pixelise) {
-        if constexpr (WIDE)
-            key = (P)loc2pix<NEST, int64_t>(g, o.dz, o.tt, o.dx, o.dy);
-        else
-#ifdef TB_X_NOPIX
-            key = (P)((int)(o.tt * 1000.0) & 0xffff);  // ablation: no HEALPix integer/floor logic
-#else
-            key = (P)loc2key32<NEST, TB_TTOFF && TB_INCR && NNZ == 3>(g, o.dz, o.tt, o.dx, o.dy);
-#endif
-    }
-    if (!ok) key = -1;
-    return key;
+    P key;
+    if constexpr (WIDE)
+        key = (P)loc2pix<NEST, int64_t>(g, o.dz, o.tt, o.dx, o.dy);
+    else
+        key = (P)loc2ckey<NEST, kOff<NNZ, P>>(g, kc, o.dz, o.tt, o.t1m, o.dx, o.dy);
+    return pixelise ? key : (P)-1;
 }
 
-// The A4 contribution of a det-sample, pending until aggregate() folds it into the run.
-// Det-flagged samples keep their key (they mark hit submaps, as A2 does) but add 0 (their
-// staged tod is 0); so does every sample without a key (aggregate() adds unconditionally).
-template <int NNZ, typename P>
-__device__ __forceinline__ void set_pending(Slot<P>& sl, const StageA& o, P key, double tod) {
-    sl.pend_key = key;
-#if TB_FOLD
-    sl.p0 = tod;
-    if (NNZ == 3) {
-        const double t = tod * o.invr;
-#else
-    sl.p0 = tod * sl.s_cal;
-    if (NNZ == 3) {
-        const double t = (tod * sl.s_eta) * o.invr;
-#endif
-        sl.p1 = t * o.cw;
-        sl.p2 = t * o.sw;
-    }
-}
-
-// One det-sample of slot `sl` with the per-sample state x.  `tod` is already 0 for det-flagged
-// samples (and, with debug outputs, shared-flagged ones): the block prologue zeroes them in the
-// staged tile, so no per-sample flag test is needed here.  Its contribution is folded into the
-// lane's run by aggregate() one sample LATER, so that work overlaps the next sample's loads.
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE>
-__device__ __forceinline__ void det_sample(Slot<typename PixT<WIDE>::T>& sl, const double* x, bool pixelise,
-                                           double tod, const HealpixGeom& g, const FusedArgs& a, int64_t d,
-                                           int64_t s) {
-    using P = typename PixT<WIDE>::T;
-    const StageA o = stage_a<NNZ, HWP, P>(sl, x);
-    const P key = stage_b<NEST, NNZ, WIDE>(o, pixelise, sl.ok, g);
-    if (DEBUG && sl.ok) {
-        const int64_t off = d * a.n_samp + s;
-        if (a.pixels_out) a.pixels_out[off] = key < 0 ? (int64_t)-1 : (int64_t)key_to_pix<NEST, WIDE>(key, g);
-        if (a.weights_out) {
-            a.weights_out[off * NNZ] = a.cal;
-            if (NNZ == 3) {
-                a.weights_out[off * NNZ + 1] = sl.etacal * (o.cw * o.invr);
-                a.weights_out[off * NNZ + 2] = sl.etacal * (o.sw * o.invr);
-            }
-        }
-    }
-    set_pending<NNZ, P>(sl, o, key, tod);
-}
-
-// Fold the pending contribution into the run (run-length aggregation along time).  Lanes
-// without a pixel (no detector / flagged sample) have pend_key = -1 and never start a run.
-// A pending sample without a pixel carries zero contributions, so the add is unconditional
-// (one branch less per det-sample); pend_key is not reset here because det_sample() always
-// overwrites it right after (the end-of-item call is followed by the final flush).  The first
-// run of an item flushes nothing: run_loc starts at -1.
-template <bool NEST, int NNZ, bool WIDE>
-__device__ __forceinline__ void aggregate(Slot<typename PixT<WIDE>::T>& sl, const FusedArgs& a,
-                                          const HealpixGeom& g, const CtaMem& cm) {
-    if (sl.pend_key >= 0 && sl.pend_key != sl.run_key) {
-#ifndef TB_X_NOFLUSH
-        flush<NNZ, WIDE>(sl, a);
-#endif
-        sl.run_key = sl.pend_key;
-        start_run<NEST, WIDE>(sl.pend_key, a, g, sl, cm);
-        sl.r0 = sl.r1 = sl.r2 = 0.0;
-    }
-    sl.r0 += sl.p0;
-    if (NNZ == 3) {
-        sl.r1 += sl.p1;
-        sl.r2 += sl.p2;
-    }
-}
-// A block of the stream: samples [s0, s0 + nb) of chunk c for detector rows d0 .. d0+nrows-1.
+// A block of the stream: samples [s0 + k0, s0 + k0 + nb) of the box starting at s0 (a multiple
+// of 16), detector rows d0 .. d0 + nrows - 1.
 struct Blk {
-    int64_t item;  // < 0: end of stream
-    int64_t d0;
-    int64_t s0;     // first sample of the staged box
-    int64_t s_end;  // end of the item's chunk
-    int nb;         // samples processed: box indices k0 .. k0 + nb - 1
+    int item;   // < 0: end of stream
+    int d0;
+    int s0;     // first sample of the staged box (multiple of 16)
+    int s_end;  // end of the item's chunk
+    int nb;     // samples processed: box indices k0 .. k0 + nb - 1
     int nrows;
-    int k0 = 0;     // TMA path: first processed box sample (boxes start at multiples of 16)
+    int k0;
 };
 
-template <int DPL>
-__device__ __forceinline__ void issue_block(RawBlock<DPL>& rb, const Blk& bk, const FusedArgs& a, bool have_dflags,
-                                            bool hwp, int lane) {
-    constexpr int kRows = 32 * DPL;
-    const int64_t n_samp = a.n_samp;
-    const int scol = lane & (kBlk - 1);
-    const int srow = lane / kBlk;
-    if (scol < bk.nb) {
-        const double* src = a.det_data + (bk.d0 + srow) * n_samp + bk.s0 + scol;
-        const int64_t step = kRowStep * n_samp;
-        const uint64_t pol = evict_first_policy();
-        if (bk.nrows == kRows) {
-#pragma unroll 8
-            for (int r = srow; r < kRows; r += kRowStep, src += step) cp_async8_stream(&rb.tod[r][scol], src, pol);
-        } else {
-            for (int r = srow; r < bk.nrows; r += kRowStep, src += step) cp_async8_stream(&rb.tod[r][scol], src, pol);
+// The lean run flush: 32-bit keys, a power-of-two submap, the cached global2local, an fp64 map,
+// no reading-R3 rotation (every map element index is < 2^31 when nside <= 4096).
+template <bool NEST, int NNZ, bool OFF>
+__device__ __forceinline__ void flush_lean(int key, double r0, double r1, double r2, const FusedArgs& a,
+                                           const HealpixGeom& g, uint16_t* g2l) {
+    const MapGeom& mg = a.map;
+    const unsigned pix = (unsigned)ckey_to_pix_bf<NEST, OFF>(key, g);
+    const unsigned sm = pix >> mg.sm_shift;
+    const unsigned lp = pix & (unsigned)(mg.n_pix_submap - 1);
+    const unsigned v = g2l[sm];
+    g2l[sm] = (uint16_t)(v | kHitBit);  // idempotent: every writer stores the same value
+    const unsigned loc = v & 0x7fffu;
+    if (loc != kNoLoc) {
+        double* dst = a.zmap + (size_t)((loc << mg.sm_shift) + lp) * NNZ;
+        red_f64(dst, r0);
+        if (NNZ == 3) {
+            red_f64(dst + 1, r1);
+            red_f64(dst + 2, r2);
         }
     }
-    // boresight: 16 quaternions = 32 x 16 B, one per lane
-    if ((lane >> 1) < bk.nb) cp_async16(&rb.bore[lane >> 1][2 * (lane & 1)], a.boresight + 4 * (bk.s0 + (lane >> 1)) + 2 * (lane & 1));
-    if (hwp && lane < bk.nb) cp_async8(&rb.hwp[lane], a.hwp + bk.s0 + lane);
-    if (a.shared_flags && lane < 5) cp_async_bytes(rb.sflg, a.shared_flags + bk.s0, bk.nb, lane);
-    if (have_dflags) {
-#pragma unroll
-        for (int j = 0; j < DPL; ++j) {
-            const int row = lane + 32 * j;
-            if (row < bk.nrows) {
-#pragma unroll
-                for (int w = 0; w < 5; ++w) cp_async_bytes(rb.flg[row], a.det_flags + (bk.d0 + row) * n_samp + bk.s0, bk.nb, w);
-            }
-        }
-    }
-    cp_async_commit();
 }
 
-// SCAN = true: the scan direction, toast_pointing_to_tod: the same item / block
-// stream, staging and per-det-sample arithmetic, but each det-sample GATHERS its pixel's map
-// values (cached per lane across the run) and updates its TOD in the staged tile; the processed
-// columns of the tile are written back after each block (per-lane stores: a TMA store of the
-// whole box would overwrite samples of a neighbouring chunk that another warp owns).
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL, bool TMA, bool SCAN = false>
-__global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_kernel(const Chunk* __restrict__ chunks,
-                                                                         int64_t n_chunks, FusedArgs a,
-                                                                         HealpixGeom g,
-                                                                         unsigned long long* __restrict__ sched,
-                                                                         const __grid_constant__ TmaMaps tm) {
-    static_assert(!TMA || (DPL == 1 && kBlk == 16), "the TMA path stages 32 x 16 tiles");
-    static_assert(!SCAN || (DPL == 1 && !DEBUG), "the scan direction: one detector per lane, no debug outputs");
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool TMA, bool SCAN>
+__global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
+    pointing_to_map_kernel(const Chunk* __restrict__ chunks, int n_chunks, FusedArgs a, HealpixGeom g, KeyConsts kc,
+                           unsigned long long* __restrict__ sched, const __grid_constant__ TmaMaps tm) {
+    static_assert(!SCAN || !DEBUG, "the scan direction has no debug outputs");
     using P = typename PixT<WIDE>::T;
+    constexpr bool OFF = kOff<NNZ, P>;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int lane = threadIdx.x & 31;
     const int wid = threadIdx.x >> 5;
-    // cp.async path: WarpSmem<DPL>; TMA path: TmaWarpSmem (1 KB-aligned, see launch_t)
-    WarpSmem<DPL>& sm = reinterpret_cast<WarpSmem<DPL>*>(smem_raw)[wid];
-    // (offset arithmetic on the __shared__ array itself, so every access below stays an LDS;
-    // the alignment that matters for TMA and the swizzle is that of the shared-window offset)
+    // the warps' areas start at the first 1 KB boundary of the shared window (the launch reserves
+    // the padding); offset arithmetic on the __shared__ array itself keeps accesses LDS / STS
     const unsigned pad1k = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
-    TmaWarpSmem& tw = reinterpret_cast<TmaWarpSmem*>(smem_raw + pad1k)[wid];
-    // the CTA's spread table and hit-submap flags: after every warp's staging area
-    unsigned char* cta_extra = smem_raw + (TMA ? 1024 + kWarps * sizeof(TmaWarpSmem) : kWarps * sizeof(WarpSmem<DPL>));
-    uint16_t* s_spread = reinterpret_cast<uint16_t*>(cta_extra);
-    uint8_t* s_hits = cta_extra + kSpreadBytes;
-    const CtaMem cm{s_spread, s_hits};
-    const bool shared_hits = a.map.shared_hits;
-    for (int i = threadIdx.x; i < 256; i += blockDim.x) {
-        unsigned v = 0u;
-        for (int b = 0; b < 8; ++b) v |= ((i >> b) & 1u) << (2 * b);
-        s_spread[i] = (uint16_t)v;
-    }
-    if (shared_hits)
-        for (int i = threadIdx.x; i < (int)a.map.n_submap; i += blockDim.x) s_hits[i] = 0;
+    WarpSmem& ws = reinterpret_cast<WarpSmem*>(smem_raw + pad1k)[wid];
+    uint16_t* s_g2l = reinterpret_cast<uint16_t*>(smem_raw + pad1k + kWarps * sizeof(WarpSmem));
+    int& s_nocache = *reinterpret_cast<int*>(smem_raw + pad1k + kWarps * sizeof(WarpSmem) +
+                                             ((2 * a.map.n_submap * a.map.cache_g2l + 15) & ~15));
+    const MapGeom& mg = a.map;
+    if (threadIdx.x == 0) s_nocache = 0;
     __syncthreads();
-    constexpr int kRows = 32 * DPL;
-    const int64_t n_groups = (a.n_det + kRows - 1) / kRows;
-    const int64_t n_items = n_chunks * n_groups;
+    if (mg.cache_g2l) {
+        for (int i = threadIdx.x; i < (int)mg.n_submap; i += blockDim.x) {
+            const int64_t v = __ldg(&mg.global2local[i]);
+            if (v >= (int64_t)kNoLoc) s_nocache = 1;  // local index beyond the 15-bit cache
+            s_g2l[i] = v < 0 ? kNoLoc : (uint16_t)(v & 0x7fff);
+        }
+    }
+    __syncthreads();
+    const CtaMem cm{s_g2l, mg.cache_g2l && !s_nocache};
+    const bool lean = !WIDE && mg.sm_shift >= 0 && cm.cached && !a.map_f32 &&
+                      !(a.gamma != nullptr && a.hwp != nullptr) && a.hit_submaps != nullptr;
+
+    const int n_groups = (int)((a.n_det + 31) / 32);
+    const int n_items = n_chunks * n_groups;
     const unsigned dmask = a.det_flag_mask;
     const unsigned smask = a.shared_flag_mask;
     const bool have_dflags = !SCAN && a.det_flags != nullptr;  // scan_map ignores det flags (S12)
     const bool have_sflags = a.shared_flags != nullptr;
+    const int n_samp = (int)a.n_samp;
     // TMA: bytes landing per block (full boxes, out-of-range elements zero-filled)
-    const unsigned tx_bytes = 32 * 16 * 8 + 16 * 32 + (have_dflags ? 32 * 16 : 0) +
-                              ((HWP && NNZ == 3) ? 16 * 8 : 0) + (have_sflags ? 16 : 0);
+    const unsigned tx_bytes = 32 * 16 * 8 + 16 * 32 + (have_dflags ? 32 * 16 : 0) + ((HWP && NNZ == 3) ? 16 * 8 : 0) +
+                              (have_sflags ? 16 : 0);
     unsigned phase = 0u;  // TMA: bit b = parity of the next completion of mbar[b]
-    const double sgn_ds = (a.should_subtract ? -1.0 : 1.0) * a.data_scale;  // SCAN only
-    const double keep_old = a.should_zero ? 0.0 : 1.0;                       // SCAN only
-    // swizzled byte offset of row `lane` in a TOD tile; sample k is at row_swz ^ (8 k)
+    const uint64_t pol = evict_first_policy();
+    // swizzled byte offset of row `lane` in a TOD tile (16-byte chunk c of row r at c ^ (r & 7));
+    // sample k is at row_swz ^ (8 k)
     const unsigned row_swz = (unsigned)lane * 128u + (((unsigned)lane & 7u) << 4);
 
-    // Lane 0 fetches the NEXT item id and its chunk descriptor one item ahead (issued at
-    // an item switch, consumed at the next one), so neither latency is on the critical path.
-    int64_t pend_item = -1, pend_first = 0;
-    int pend_count = 0;
+    // Lane 0 fetches the NEXT item id and its chunk descriptor one item ahead (issued at an item
+    // switch, consumed at the next one), so neither latency is on the critical path.
+    int pend_item = -1, pend_first = 0, pend_count = 0;
     auto prefetch_item = [&]() {
         if (lane == 0) {
             const unsigned long long it = atomicAdd(sched, 1ull);
-            pend_item = it < (unsigned long long)n_items ? (int64_t)it : -1;
+            pend_item = it < (unsigned long long)n_items ? (int)it : -1;
             if (pend_item >= 0) {
                 const Chunk ch = chunks[pend_item / n_groups];
-                pend_first = ch.first;
+                pend_first = (int)ch.first;
                 pend_count = ch.count;
             }
         }
     };
     auto take_item = [&]() -> Blk {
         Blk bk;
-        bk.item = __shfl_sync(0xffffffffu, pend_item, 0);
-        const int64_t first = __shfl_sync(0xffffffffu, pend_first, 0);
-        const int count = __shfl_sync(0xffffffffu, pend_count, 0);
+        bk.item = __shfl_sync(kFull, pend_item, 0);
+        const int first = __shfl_sync(kFull, pend_first, 0);
+        const int count = __shfl_sync(kFull, pend_count, 0);
         if (bk.item < 0) {
-            bk.d0 = bk.s0 = bk.s_end = 0;
-            bk.nb = bk.nrows = 0;
+            bk.d0 = bk.s0 = bk.s_end = bk.nb = bk.nrows = bk.k0 = 0;
             return bk;
         }
-        const int64_t c = bk.item / n_groups;
-        bk.d0 = (bk.item - c * n_groups) * kRows;
-        bk.nrows = (a.n_det - bk.d0) < kRows ? (int)(a.n_det - bk.d0) : kRows;
-        bk.s0 = first;
+        const int c = bk.item / n_groups;
+        bk.d0 = (bk.item - c * n_groups) * 32;
+        bk.nrows = min(32, (int)a.n_det - bk.d0);
+        // boxes start at multiples of 16 samples (a TMA box must start 16-byte aligned in every
+        // staged row; the u8 flag rows need that); a chunk's first block processes k0 .. 15 only
+        bk.k0 = first & 15;
+        bk.s0 = first - bk.k0;
         bk.s_end = first + count;
-        bk.nb = count < kBlk ? count : kBlk;
-        if (TMA) {
-            // TMA boxes must start on 16-byte boundaries of every staged row (measured: an odd
-            // f64 start faults), so boxes are aligned to 16 samples — the u8 flag rows need
-            // that — and a chunk's first block processes box samples k0 .. 15 only
-            bk.k0 = (int)(first & 15);
-            bk.s0 = first - bk.k0;
-            bk.nb = count < kBlk - bk.k0 ? count : kBlk - bk.k0;
-        }
+        bk.nb = min(count, kBlk - bk.k0);
         return bk;
+    };
+    auto successor = [&](const Blk& cur) -> Blk {
+        Blk nx;
+        if (cur.s0 + kBlk < cur.s_end) {
+            nx = cur;
+            nx.s0 = cur.s0 + kBlk;
+            nx.k0 = 0;
+            nx.nb = min(kBlk, nx.s_end - nx.s0);
+        } else {
+            nx = take_item();
+            if (nx.item >= 0) prefetch_item();
+        }
+        return nx;
     };
     // Stage the raw inputs of block bk into buffer b.
     auto issue = [&](int b, const Blk& bk) {
@@ -721,284 +584,288 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
                 // the generic-proxy reads of buffer b (two blocks ago) are ordered before the
                 // async-proxy writes that refill it
                 asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
-                mbar_expect_tx(&tw.sf[b].mbar, tx_bytes);
-                const uint64_t pol = evict_first_policy();
-                const int s0 = (int)bk.s0, d0 = (int)bk.d0;
-                tma_2d_stream(&tw.tod[b][0][0], &tm.tod, s0, d0, &tw.sf[b].mbar, pol);
-                if (have_dflags) tma_2d_stream(&tw.flg[b][0][0], &tm.flg, s0, d0, &tw.sf[b].mbar, pol);
-                tma_2d(&tw.bore[b][0][0], &tm.bore, 0, s0, &tw.sf[b].mbar);
-                if (HWP && NNZ == 3) tma_1d(&tw.hwp[b][0], &tm.hwp, s0, &tw.sf[b].mbar);
-                if (have_sflags) tma_1d(&tw.sf[b].f[0], &tm.sflg, s0, &tw.sf[b].mbar);
+                mbar_expect_tx(&ws.sf[b].mbar, tx_bytes);
+                tma_2d_stream(&ws.tod[b][0][0], &tm.tod, bk.s0, bk.d0, &ws.sf[b].mbar, pol);
+                if (have_dflags) tma_2d_stream(&ws.flg[b][0][0], &tm.flg, bk.s0, bk.d0, &ws.sf[b].mbar, pol);
+                tma_2d(&ws.bore[b][0][0], &tm.bore, 0, bk.s0, &ws.sf[b].mbar);
+                if (HWP && NNZ == 3) tma_1d(&ws.hwp[b][0], &tm.hwp, bk.s0, &ws.sf[b].mbar);
+                if (have_sflags) tma_1d(&ws.sf[b].f[0], &tm.sflg, bk.s0, &ws.sf[b].mbar);
             }
         } else {
-            issue_block<DPL>(sm.buf[b], bk, a, have_dflags, HWP && NNZ == 3, lane);
+            // per-lane cp.async into the same (swizzled) layout; only the block's own samples
+            const int scol = lane & 15, srow = lane >> 4;
+            const bool valid = scol >= bk.k0 && scol < bk.k0 + bk.nb;
+            if (valid) {
+                const double* src = a.det_data + (int64_t)(bk.d0 + srow) * n_samp + bk.s0 + scol;
+                const unsigned base = smem_u32(&ws.tod[b][0][0]);
+                for (int r = srow; r < bk.nrows; r += 2, src += 2 * (int64_t)n_samp)
+                    cp_async8_pol(base + (unsigned)r * 128u + (((unsigned)scol << 3) ^ (((unsigned)r & 7u) << 4)), src,
+                                  pol);
+            }
+            if ((lane >> 1) >= bk.k0 && (lane >> 1) < bk.k0 + bk.nb)
+                cp_async16(&ws.bore[b][lane >> 1][2 * (lane & 1)],
+                           a.boresight + 4 * (int64_t)(bk.s0 + (lane >> 1)) + 2 * (lane & 1));
+            if (HWP && NNZ == 3 && valid && lane < 16) cp_async8(smem_u32(&ws.hwp[b][lane]), a.hwp + bk.s0 + lane);
+            cp_async_commit();
+            // flags: plain loads of the block's own bytes (the rows need not be 4-byte aligned)
+            if (have_sflags && valid && lane < 16) ws.sf[b].f[lane] = __ldg(a.shared_flags + bk.s0 + lane);
+            if (have_dflags && lane < bk.nrows) {
+                const uint8_t* fr = a.det_flags + (int64_t)(bk.d0 + lane) * n_samp + bk.s0;
+                for (int k = bk.k0; k < bk.k0 + bk.nb; ++k) ws.flg[b][lane][k] = __ldg(fr + k);
+            }
         }
     };
 
     if constexpr (TMA) {
         if (lane == 0) {
-            mbar_init(&tw.sf[0].mbar);
-            mbar_init(&tw.sf[1].mbar);
+            mbar_init(&ws.sf[0].mbar);
+            mbar_init(&ws.sf[1].mbar);
             asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
         }
         __syncwarp();
     }
     prefetch_item();
     Blk cur = take_item();
-    // every thread reaches the shared-hits flush below (a warp without work skips the stream)
+    // every thread reaches the hit-flag write-back below (a warp without work skips the stream)
     if (cur.item >= 0) [&] {
         prefetch_item();
         issue(0, cur);
-        Slot<P> sl[DPL];
-#pragma unroll
-        for (int j = 0; j < DPL; ++j) load_slot<P>(sl[j], a, cur.d0 + lane + 32 * j, lane + 32 * j < cur.nrows, cur.d0);
-        int p = 0;
+        Slot<P> sl;
+        load_slot<P>(sl, a, cur.d0 + lane, lane < cur.nrows, cur.d0);
+        const double sgn_ds = (a.should_subtract ? -1.0 : 1.0) * a.data_scale;  // SCAN only
 
+        // A run ends: flush it (the lanes whose key changed; divergent).
+        auto flush_run = [&]() {
+            if (lean) {
+                flush_lean<NEST, NNZ, OFF>((int)sl.run_key, sl.r0 * sl.sI, sl.r1 * sl.sQ, sl.r2 * sl.sU, a, g, cm.g2l);
+            } else {
+                drain_general<NEST, NNZ, OFF, WIDE>(sl.run_key, sl.r0 * sl.sI, sl.r1 * sl.sQ, sl.r2 * sl.sU, a.zmap,
+                                                    a.map_f32, a.hit_submaps, mg.global2local, mg.sm_shift,
+                                                    mg.n_pix_submap, cm.g2l, cm.cached, a.gamma, a.hwp != nullptr,
+                                                    a.iau, sl.det, g);
+            }
+        };
+
+        int p = 0;
         while (true) {
             // successor block: next 16 samples of this item, or the first block of the next item
-            Blk nxt;
-            if (cur.s0 + kBlk < cur.s_end) {
-                nxt = cur;
-                nxt.s0 = cur.s0 + kBlk;
-                nxt.k0 = 0;
-                nxt.nb = (nxt.s_end - nxt.s0) < kBlk ? (int)(nxt.s_end - nxt.s0) : kBlk;
-            } else {
-                nxt = take_item();
-                if (nxt.item >= 0) prefetch_item();
-            }
+            const Blk nxt = successor(cur);
             if constexpr (TMA) {
-                mbar_wait(&tw.sf[p].mbar, (phase >> p) & 1u);
+                mbar_wait(&ws.sf[p].mbar, (phase >> p) & 1u);
                 phase ^= 1u << p;
             } else {
                 cp_async_wait_all();
                 __syncwarp();
             }
             if (nxt.item >= 0) issue(p ^ 1, nxt);
-            __syncwarp();  // reconverge after the lane-0 / spin-wait paths (else the state code below runs twice)
-
-            RawBlock<DPL>& rb = sm.buf[p];
-            // Per-sample state, split over the warp: lanes 0..kBlk-1 build the boresight rotation
-            // matrix of sample `lane` (identity if shared-flagged, S2), lanes 16..16+kBlk-1 the HWP
-            // cos/sin(4 chi) of sample `lane - 16`.  Bit k of pmask = sample k is pixelised.
-            double* st_base = TMA ? &tw.st[0][0] : &sm.st[0].v[0];
+            __syncwarp();  // reconverge after the lane-0 / spin-wait paths
+            double* st_base = &ws.st[0][0];
             bool pixelise_me = false;
             {
+                // lanes 0..15: the boresight rotation matrix of sample `lane` (identity if
+                // shared-flagged, S2); lanes 16..31: the HWP cos/sin(4 chi) of sample `lane - 16`
                 const int ks = lane & 15;
-                const bool in_blk = ks < kBlk && ks >= cur.k0 && ks < cur.k0 + cur.nb;
+                const bool in_blk = ks >= cur.k0 && ks < cur.k0 + cur.nb;
                 if (lane < kBlk) {
                     double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 1.0;
                     if (in_blk) {
-                        bool flagged;
-                        if constexpr (TMA) {
-                            flagged = have_sflags && (tw.sf[p].f[lane] & smask);
-                        } else {
-                            const int soff =
-                                have_sflags ? (int)(reinterpret_cast<uintptr_t>(a.shared_flags + cur.s0) & 3) : 0;
-                            flagged = have_sflags && (rb.sflg[soff + lane] & smask);
-                        }
+                        const bool flagged = have_sflags && (ws.sf[p].f[lane] & smask);
                         pixelise_me = !flagged;
-                        const double* bq = TMA ? tw.bore[p][lane] : rb.bore[lane];
                         if (!flagged) {
+                            const double* bq = ws.bore[p][lane];
                             q0 = bq[0]; q1 = bq[1]; q2 = bq[2]; q3 = bq[3];
                         }
                     }
-                    double m[10];
+                    double m[9];
                     quat_to_matrix(q0, q1, q2, q3, m);
-                    m[9] = 1.0;
                     double2* dst = reinterpret_cast<double2*>(st_base + 12 * lane);
 #pragma unroll
                     for (int i = 0; i < 4; ++i) dst[i] = make_double2(m[2 * i], m[2 * i + 1]);
                     st_base[12 * lane + 8] = m[8];
-                } else if (HWP && NNZ == 3 && ks < kBlk) {
+                } else if (HWP && NNZ == 3) {
                     double c4 = 1.0, s4 = 0.0;
-                    if (in_blk) small_sincos(4.0 * (TMA ? tw.hwp[p][ks] : rb.hwp[ks]), &s4, &c4);
+                    if (in_blk) {
+                        // reading R1: any finite chi; the Cody-Waite reduction of small_sincos
+                        // holds for |4 chi| < 2^20 pi/2, CUDA's full-range sincos beyond
+                        const double a4 = 4.0 * ws.hwp[p][ks];
+                        if (fabs(a4) < 1.6e6)
+                            small_sincos(a4, &s4, &c4);
+                        else
+                            sincos(a4, &s4, &c4);
+                    }
                     st_base[12 * ks + 9] = c4;
-                    st_base[12 * ks + 10] = s4;
+                    st_base[12 * ks + 10] = 2.0 * s4;
+                    st_base[12 * ks + 11] = 0.5 * s4;
                 }
             }
-            const unsigned pmask = __ballot_sync(0xffffffffu, pixelise_me);
-            const unsigned keep = ((1u << cur.nb) - 1u) << cur.k0;  // samples of the block processed (nb <= 16)
-            // The staged TOD of det-flagged samples (and, with debug outputs, of shared-flagged
-            // samples, which run through det_sample without a pixel) is zeroed in shared memory, so
-            // the per-sample loop needs no flag test: those samples add exactly 0 to the map.
+            const unsigned pmask = __ballot_sync(kFull, pixelise_me) & 0xffffu;
+            const unsigned keep = ((1u << cur.nb) - 1u) << cur.k0;  // samples of the block processed
+            // zm: samples whose staged TOD is zeroed — det-flagged (they add exactly 0 but still
+            // form runs and mark their submap, reading R2) and, in the map direction,
+            // shared-flagged ones (they run through the loop with key -1)
+            unsigned zm = SCAN ? 0u : (~pmask & keep);
+            if (have_dflags && lane < cur.nrows) {
+                const uint4 f = *reinterpret_cast<const uint4*>(ws.flg[p][lane]);
+                const unsigned rep = dmask * 0x01010101u;
+                const unsigned fw[4] = {f.x & rep, f.y & rep, f.z & rep, f.w & rep};
+                if (fw[0] | fw[1] | fw[2] | fw[3]) {  // rare: 16 samples of 1 % flags
 #pragma unroll
-            for (int j = 0; j < DPL; ++j) {
-                const int row = lane + 32 * j;
-                unsigned zm = DEBUG ? (~pmask & keep) : 0u;
-                if (have_dflags && row < cur.nrows) {
-                    const unsigned rep = dmask * 0x01010101u;
-                    unsigned bits = 0u;  // bit k: sample k of the box is det-flagged
-                    if constexpr (TMA) {
-                        const uint4 f = *reinterpret_cast<const uint4*>(tw.flg[p][row]);
-                        const unsigned fw[4] = {f.x, f.y, f.z, f.w};
+                    for (int w = 0; w < 4; ++w)
 #pragma unroll
-                        for (int w = 0; w < 4; ++w) {
-                            const unsigned v = __vcmpne4(fw[w] & rep, 0u);
-                            bits |= ((v & 0x01010101u) * 0x01020408u >> 24 & 0xfu) << (4 * w);
-                        }
-                    } else {
-                        const int foff =
-                            (int)(reinterpret_cast<uintptr_t>(a.det_flags + (cur.d0 + row) * a.n_samp + cur.s0) & 3);
-#pragma unroll
-                        for (int w = 0; w < 5; ++w) {  // bit b: byte b of the 20-byte window is flagged
-                            const unsigned v = __vcmpne4(*reinterpret_cast<const unsigned*>(&rb.flg[row][4 * w]) & rep, 0u);
-                            bits |= ((v & 0x01010101u) * 0x01020408u >> 24 & 0xfu) << (4 * w);
-                        }
-                        bits >>= foff;
-                    }
-                    zm |= bits & keep;
+                        for (int b = 0; b < 4; ++b)
+                            if ((fw[w] >> (8 * b)) & 0xffu) zm |= 1u << (4 * w + b);
                 }
-                while (zm) {
-                    const int k = __ffs(zm) - 1;
-                    zm &= zm - 1;
-                    if constexpr (TMA)
-                        *reinterpret_cast<double*>(reinterpret_cast<unsigned char*>(&tw.tod[p][0][0]) +
-                                                   (row_swz ^ ((unsigned)k << 3))) = 0.0;
-                    else
-                        rb.tod[row][k] = 0.0;
+                zm &= keep;
+            }
+            {
+                const unsigned tile0 = smem_u32(&ws.tod[p][0][0]) + row_swz;
+                unsigned z = zm;
+                while (z) {
+                    const int c = __ffs(z) - 1;
+                    z &= z - 1;
+                    asm volatile("st.shared.f64 [%0], %1;" ::"r"(tile0 ^ ((unsigned)c << 3)), "d"(0.0) : "memory");
                 }
             }
             __syncwarp();
 
-            // TMA tile: the tile is 1 KB-aligned and row r starts at r * 128, so the swizzled address
-            // of (lane, k) is (tile + row_swz) ^ (8 k): one LOP3 per sample.
-            const unsigned tod_row = smem_u32(&tw.tod[p][0][0]) + row_swz;
-            // SCAN: the per-lane gather cache lives in the slot (run_key / run_loc: the cached
-            // pixel's key and storage; r0..r2 its map values; pend_key: the block sample whose TOD
-            // update waits for them, completed one sample later so the gather latency hides
-            // behind that sample)
-            auto store_tod = [&](int kk, double v) {
-                if constexpr (TMA)
-                    asm volatile("st.shared.f64 [%0], %1;" ::"r"(tod_row ^ ((unsigned)kk << 3)), "d"(v) : "memory");
-                else
-                    rb.tod[lane][kk] = v;
-            };
-            auto scan_finish = [&]() {
-                if constexpr (SCAN) {
-                    Slot<P>& s0 = sl[0];
-                    if (s0.pend_key >= 0) {
-                        double t = s0.r0 * a.cal;
-                        if (NNZ == 3) t += s0.etacal * (s0.r1 * s0.p1 + s0.r2 * s0.p2);
-                        store_tod((int)s0.pend_key, fma(sgn_ds, t, keep_old * s0.p0));
-                        s0.pend_key = -1;
-                    }
-                }
-            };
-            auto scan_sample = [&](int kk, const double* x, double tod) {
-                if constexpr (SCAN) {
-                    Slot<P>& s0 = sl[0];
-                    const StageA o = stage_a<NNZ, HWP, P>(s0, x);
-                    const P key = stage_b<NEST, NNZ, WIDE>(o, true, s0.ok, g);
-                    scan_finish();  // the previous sample's gathered values have arrived by now
-                    const MapGeom& mg = a.map;
-                    if (key >= 0 && key != s0.run_key) {
-                        P pix;
-                        if constexpr (WIDE)
-                            pix = key;
-                        else
-                            pix = key_to_pix_tab<NEST>(key, g, cm.spread);
-                        const int64_t smi = submap_of<P>(pix, mg);
-                        if (smi != (int64_t)s0.last_sm) {
-                            s0.last_loc = __ldg(&mg.global2local[smi]);
-                            s0.last_sm = (P)smi;
-                        }
-                        s0.run_key = key;
-                        s0.run_loc = s0.last_loc;
-                        if (s0.run_loc >= 0) {
-                            const int64_t lp = mg.sm_shift >= 0 ? (int64_t)(pix & (P)(mg.n_pix_submap - 1))
-                                                                : (int64_t)pix - smi * mg.n_pix_submap;
-                            const double* mp = a.mapdata + (s0.run_loc * mg.n_pix_submap + lp) * NNZ;
-                            s0.r0 = __ldg(mp);
-                            if (NNZ == 3) {
-                                s0.r1 = __ldg(mp + 1);
-                                s0.r2 = __ldg(mp + 2);
-                            }
-                        }
-                    }
-                    if (key >= 0 && s0.run_loc >= 0) {
-                        s0.pend_key = (P)kk;
-                        s0.p0 = tod;
-                        s0.p1 = o.cw * o.invr;
-                        s0.p2 = o.sw * o.invr;
-                    }
-                }
-            };
-
-            int k = cur.k0;
-            const int k_end = cur.k0 + cur.nb;
-            unsigned bit = 1u << k;  // 1 << k
-#pragma unroll kKUnroll
-            for (; k < k_end; ++k, bit <<= 1) {
-                const bool pixelise = pmask & bit;
-                if (!DEBUG && !pixelise) continue;  // shared-flagged sample: nothing to add (uniform)
-                double x[12];
+            auto load_state = [&](int k, double* x) {
 #pragma unroll
                 for (int i = 0; i < ((HWP && NNZ == 3) ? 12 : 10); i += 2) {
                     const double2 t2 = *reinterpret_cast<const double2*>(st_base + 12 * k + i);
                     x[i] = t2.x;
                     x[i + 1] = t2.y;
                 }
-                double tod[DPL];
-#pragma unroll
-                for (int j = 0; j < DPL; ++j) {
-                    if constexpr (TMA)
-                        asm volatile("ld.shared.f64 %0, [%1];" : "=d"(tod[j]) : "r"(tod_row ^ ((unsigned)k << 3)));
-                    else
-                        tod[j] = rb.tod[lane + 32 * j][k];
-                }
-                if constexpr (SCAN) {
-                    scan_sample(k, x, tod[0]);
-                } else {
-#if TB_DEFER
-                    // fold the previous sample while those shared-memory loads are in flight
-#pragma unroll
-                    for (int j = 0; j < DPL; ++j) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, cm);
-#endif
-#pragma unroll
-                    for (int j = 0; j < DPL; ++j)
-                        det_sample<NEST, NNZ, HWP, DEBUG, WIDE>(sl[j], x, pixelise, tod[j], g, a,
-                                                                cur.d0 + lane + 32 * j, cur.s0 + k);
-#if !TB_DEFER
-                    // fold this sample at once: no pending contribution is carried across iterations
-#pragma unroll
-                    for (int j = 0; j < DPL; ++j) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, cm);
-#endif
-                }
-            }
-            if constexpr (SCAN) {
-                scan_finish();
-                __syncwarp();
-                // write back the processed columns of the tile (two rows per warp instruction,
-                // coalesced along samples); unprocessed samples in them keep the value read
-                const int scol = lane & 15, srow = lane >> 4;
-                if (scol >= cur.k0 && scol < cur.k0 + cur.nb) {
-                    double* dst = a.tod_out + (cur.d0 + srow) * a.n_samp + cur.s0 + scol;
-                    for (int r = srow; r < cur.nrows; r += 2, dst += 2 * a.n_samp) {
+            };
+
+            // TOD tile: 1 KB-aligned, row r at r * 128, so the swizzled address of (lane, k) is
+            // (tile + row_swz) ^ (8 k): one LOP3 per sample
+            const unsigned tile = smem_u32(&ws.tod[p][0][0]) + row_swz;
+            {
+                const int kb = cur.k0, ke = cur.k0 + cur.nb;
+#pragma unroll 1
+                for (int k = kb; k < ke; ++k) {
+                    const bool pixelise = (pmask >> k) & 1u;
+                    const unsigned addr = tile ^ ((unsigned)k << 3);
+                    double x[12];
+                    load_state(k, x);
+                    const StageA o = stage_a<NNZ, HWP, P>(sl, x, kc);
+                    P key = stage_b<NEST, NNZ, WIDE>(o, pixelise, g, kc);
+                    if (!sl.ok) key = -1;
+                    if constexpr (SCAN) {
+                        // gather the run's map values (cached per lane across the run), update the TOD
+                        if (key < 0) continue;
+                        if (key != sl.run_key) {
+                            sl.run_key = key;
+                            sl.run_elem = locate(key_to_pixel<NEST, OFF, WIDE>(key, g), a, cm);
+                            if (sl.run_elem >= 0) {
+                                double m0, m1 = 0.0, m2 = 0.0;
+                                if (a.map_f32) {
+                                    const float* mp = reinterpret_cast<const float*>(a.mapdata) + sl.run_elem * NNZ;
+                                    m0 = __ldg(mp);
+                                    if (NNZ == 3) {
+                                        m1 = __ldg(mp + 1);
+                                        m2 = __ldg(mp + 2);
+                                    }
+                                } else {
+                                    const double* mp = a.mapdata + sl.run_elem * NNZ;
+                                    m0 = __ldg(mp);
+                                    if (NNZ == 3) {
+                                        m1 = __ldg(mp + 1);
+                                        m2 = __ldg(mp + 2);
+                                    }
+                                }
+                                // fold the reading-R3 rotation / IAU sign into the gathered (m1, m2)
+                                if (NNZ == 3) {
+                                    if (a.iau) m2 = -m2;
+                                    if (a.gamma != nullptr && a.hwp != nullptr) {
+                                        // t = m . (D R(-4 gamma) w) = (R(4 gamma) D m) . w; gamma_rotate
+                                        // gives diag(1, -1) R(-4 gamma) (m1, -m2) = R(4 gamma) (m1, m2)
+                                        const double2 n = gamma_rotate(m1, -m2, a.gamma, 1, sl.det);
+                                        m1 = n.x;
+                                        m2 = n.y;
+                                    }
+                                }
+                                sl.r0 = m0 * a.cal;
+                                sl.r1 = m1 * sl.etacal;
+                                sl.r2 = m2 * (2.0 * sl.etacal);
+                            }
+                        }
+                        if (sl.run_elem < 0) continue;
+                        double t = sl.r0;
+                        if (NNZ == 3) t = fma(sl.r1 * o.invr, o.cw, fma(sl.r2 * o.invr, o.sw, t));
                         double v;
-                        if constexpr (TMA)
+                        if (a.should_zero) {
+                            v = sgn_ds * t;  // the old value is overwritten, never read (NaN-safe)
+                        } else {
+                            double old;
+                            asm volatile("ld.shared.f64 %0, [%1];" : "=d"(old) : "r"(addr));
+                            v = fma(sgn_ds, t, old);
+                        }
+                        asm volatile("st.shared.f64 [%0], %1;" ::"r"(addr), "d"(v) : "memory");
+                    } else {
+                        double tod;
+                        asm volatile("ld.shared.f64 %0, [%1];" : "=d"(tod) : "r"(addr));
+                        if (DEBUG && sl.ok) {
+                            const int64_t off = sl.det * a.n_samp + cur.s0 + k;
+                            const int64_t pix = key < 0 ? -1 : key_to_pixel<NEST, OFF, WIDE>(key, g);
+                            if (a.pixels_out) a.pixels_out[off] = pix;
+                            if (a.weights_out) {
+                                a.weights_out[off * NNZ] = a.cal;
+                                if (NNZ == 3) {
+                                    double w1 = sl.etacal * (o.cw * o.invr), w2 = sl.etacal * (2.0 * o.sw * o.invr);
+                                    if (a.gamma != nullptr && a.hwp != nullptr) {
+                                        const double2 v = gamma_rotate(w1, w2, a.gamma, 0, sl.det);
+                                        w1 = v.x;
+                                        w2 = v.y;
+                                    }
+                                    a.weights_out[off * NNZ + 1] = w1;
+                                    a.weights_out[off * NNZ + 2] = a.iau ? -w2 : w2;
+                                }
+                            }
+                            if (a.dropped && pix >= 0 && !(a.det_flags && (a.det_flags[off] & dmask))) {
+                                const int64_t smi = pix / mg.n_pix_submap;
+                                if (__ldg(&mg.global2local[smi]) < 0) atomicAdd(a.dropped, 1ull);
+                            }
+                        }
+                        // run-length aggregation: the run ends when the key changes
+                        if (key != sl.run_key) {
+                            if (sl.run_key >= 0) flush_run();
+                            sl.run_key = key;
+                            sl.r0 = sl.r1 = sl.r2 = 0.0;
+                        }
+                        sl.r0 += tod;
+                        if (NNZ == 3) {
+                            const double t = tod * o.invr;
+                            sl.r1 = fma(t, o.cw, sl.r1);
+                            sl.r2 = fma(t, o.sw, sl.r2);
+                        }
+                    }
+                }
+                __syncwarp();
+                if constexpr (SCAN) {
+                    // write back the processed columns of the tile (two rows per warp instruction,
+                    // coalesced along samples); unprocessed samples in them keep the value read
+                    const int scol = lane & 15, srow = lane >> 4;
+                    if (scol >= cur.k0 && scol < cur.k0 + cur.nb) {
+                        double* dst = a.tod_out + (int64_t)(cur.d0 + srow) * n_samp + cur.s0 + scol;
+                        for (int r = srow; r < cur.nrows; r += 2, dst += 2 * (int64_t)n_samp) {
+                            double v;
                             asm volatile("ld.shared.f64 %0, [%1];"
                                          : "=d"(v)
-                                         : "r"(smem_u32(&tw.tod[p][0][0]) + (unsigned)r * 128u +
+                                         : "r"(smem_u32(&ws.tod[p][0][0]) + (unsigned)r * 128u +
                                                (((unsigned)scol << 3) ^ (((unsigned)r & 7u) << 4))));
-                        else
-                            v = rb.tod[r][scol];
-                        *dst = v;
+                            *dst = v;
+                        }
                     }
                 }
             }
 
             if (nxt.item != cur.item) {
-#pragma unroll
-                for (int j = 0; j < DPL; ++j) {
-                    if constexpr (!SCAN) {
-                        if (TB_DEFER) aggregate<NEST, NNZ, WIDE>(sl[j], a, g, cm);
-                        flush<NNZ, WIDE>(sl[j], a);
-                    }
+                if constexpr (!SCAN) {
+                    if (sl.run_key >= 0) flush_run();  // the item's open runs
                 }
                 if (nxt.item < 0) break;
-#pragma unroll
-                for (int j = 0; j < DPL; ++j)
-                    load_slot<P>(sl[j], a, nxt.d0 + lane + 32 * j, lane + 32 * j < nxt.nrows, nxt.d0);
+                load_slot<P>(sl, a, nxt.d0 + lane, lane < nxt.nrows, nxt.d0);
             }
             __syncwarp();  // all lanes are done with buffer p and st before they are refilled
             cur = nxt;
@@ -1006,10 +873,10 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB) pointing_to_map_ke
         }
         if constexpr (!TMA) cp_async_wait_all();
     }();
-    if (shared_hits) {  // the CTA's hit flags, once: a few hundred stores instead of one per run
+    if (a.hit_submaps && cm.cached) {  // the CTA's hit flags, once: a few hundred stores instead of one per run
         __syncthreads();
-        for (int i = threadIdx.x; i < (int)a.map.n_submap; i += blockDim.x)
-            if (s_hits[i]) a.hit_submaps[i] = 1;
+        for (int i = threadIdx.x; i < (int)mg.n_submap; i += blockDim.x)
+            if (s_g2l[i] & kHitBit) a.hit_submaps[i] = 1;
     }
 }
 
@@ -1039,9 +906,9 @@ bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 
 
 const cuuint64_t kNoStrides[1] = {0};  // rank-1 maps have no strides (a non-null array is passed anyway)
 
-// The TMA path applies when every staged array is 16-byte aligned, rows of the TOD and the
-// det flags are multiples of 16 bytes (n_samp % 16 == 0) and sample / detector coordinates
-// fit the 32-bit TMA coordinates; otherwise the cp.async path runs (same results).
+// The TMA path applies when every staged array is 16-byte aligned and rows of the TOD and the
+// det flags are multiples of 16 bytes (n_samp % 16 == 0); otherwise the cp.async path runs (same
+// results).
 thread_local const char* t_fused_path = "";
 
 bool make_tma_maps(const FusedArgs& a, TmaMaps* tm) {
@@ -1053,8 +920,8 @@ bool make_tma_maps(const FusedArgs& a, TmaMaps* tm) {
         t_fused_path = "cp.async (no cuTensorMapEncodeTiled)";
         return false;
     }
-    if (a.n_samp % 16 != 0 || a.n_samp >= (int64_t(1) << 31) || a.n_det >= (int64_t(1) << 31)) {
-        t_fused_path = "cp.async (n_samp % 16 != 0 or sizes beyond 32-bit TMA coordinates)";
+    if (a.n_samp % 16 != 0) {
+        t_fused_path = "cp.async (n_samp % 16 != 0)";
         return false;
     }
     if (!aligned16(a.det_data) || !aligned16(a.boresight) || (a.det_flags && !aligned16(a.det_flags)) ||
@@ -1103,80 +970,106 @@ bool make_tma_maps(const FusedArgs& a, TmaMaps* tm) {
     return true;
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL, bool TMA, bool SCAN = false>
+// Dynamic shared memory of the fused kernel: 1 KB alignment slack, the warps' areas, the
+// global2local cache and the cache-overflow flag.
+size_t fused_smem(const FusedArgs& a) {
+    return 1024 + sizeof(WarpSmem) * kWarps + ((2 * (size_t)a.map.n_submap * a.map.cache_g2l + 15) & ~size_t(15)) + 16;
+}
+
+// The dynamic shared-memory limit is a per-context attribute: raised to the opt-in maximum once
+// per device (per kernel instantiation; the statics are per template instance).
+template <typename K>
+void raise_smem_limit(K kern, bool* done_per_dev) {
+    static std::mutex mu;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) dev = 0;
+    std::lock_guard<std::mutex> lk(mu);
+    if (!done_per_dev[dev]) {
+        int optin = 0;
+        cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, optin > 0 ? optin : 232448);
+        cudaGetLastError();
+        done_per_dev[dev] = true;
+    }
+}
+
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool TMA, bool SCAN>
 cudaError_t launch_k(const WorkList& wl, const FusedArgs& a, const TmaMaps& tm, unsigned long long* sched,
                      cudaStream_t st) {
-    auto kern = pointing_to_map_kernel<NEST, NNZ, HWP, DEBUG, WIDE, DPL, TMA, SCAN>;
-    const size_t smem =
-        (TMA ? sizeof(TmaWarpSmem) * kWarps + 1024 : sizeof(WarpSmem<DPL>) * kWarps) + kSpreadBytes + kSharedHitBytes;
-    static int blocks_per_sm = 0;
-    static std::once_flag once;
-    std::call_once(once, [&] {
-        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, kern, kWarps * 32, smem) != cudaSuccess ||
-            blocks_per_sm < 1)
-            blocks_per_sm = 1;
-    });
-    const int64_t n_items = wl.n_chunks * ((a.n_det + 32 * DPL - 1) / (32 * DPL));
+    auto kern = pointing_to_map_kernel<NEST, NNZ, HWP, DEBUG, WIDE, TMA, SCAN>;
+    static bool done[64] = {false};
+    raise_smem_limit(kern, done);
+    const size_t smem = fused_smem(a);
+    // resident CTAs per SM: registers are bounded for TB_FUSED_MINB (launch bounds); shared
+    // memory decides below that (228 KB per SM, 1 KB reserved per CTA)
+    int dev = 0, smem_sm = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev);
+    int bps = smem_sm > 0 ? (int)((size_t)smem_sm / (smem + 1024)) : 1;
+    bps = std::max(1, std::min(bps, TB_FUSED_MINB));
+#ifdef TB_BPS_ENV
+    if (const char* e = getenv("TB_BPS")) bps = std::max(1, std::min(bps, atoi(e)));  // tuning experiments only
+#endif
+    const int64_t n_items = wl.n_chunks * ((a.n_det + 31) / 32);
     const int64_t want = (n_items + kWarps - 1) / kWarps;
-    const int64_t grid = std::min<int64_t>(want, (int64_t)num_sms() * blocks_per_sm);
+    const int64_t grid = std::min<int64_t>(want, (int64_t)num_sms() * bps);
     if (grid <= 0) return cudaSuccess;
     cudaError_t e = cudaMemsetAsync(sched, 0, sizeof(unsigned long long), st);
     if (e != cudaSuccess) return e;
-    kern<<<(unsigned)grid, kWarps * 32, smem, st>>>(wl.chunks, wl.n_chunks, a, make_geom(a.nside), sched, tm);
+    kern<<<(unsigned)grid, kWarps * 32, smem, st>>>(wl.chunks, (int)wl.n_chunks, a, make_geom(a.nside),
+                                                    make_key_consts(a.nside), sched, tm);
     return cudaGetLastError();
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, int DPL, bool SCAN = false>
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool SCAN>
 cudaError_t launch_t(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
     TmaMaps tm;
-    if constexpr (kBlk == 16) {
-        if (DPL == 1 && make_tma_maps(a, &tm)) {
-            t_fused_path = "tma";
-            return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, 1, true, SCAN>(wl, a, tm, sched, st);
-        }
-    } else {
-        t_fused_path = "cp.async (8-sample blocks)";
+    if (make_tma_maps(a, &tm)) {
+        t_fused_path = "tma";
+        return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, true, SCAN>(wl, a, tm, sched, st);
     }
     std::memset(&tm, 0, sizeof(tm));
-    return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, DPL, false, SCAN>(wl, a, tm, sched, st);
+    return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, false, SCAN>(wl, a, tm, sched, st);
 }
+
+// nside <= 4096: 32-bit compact keys; beyond: 64-bit pixel keys
+constexpr int64_t kCompactMaxNside = 4096;
 
 template <bool NEST, int NNZ, bool HWP, bool DEBUG>
 cudaError_t dispatch_shape(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
-    const bool wide = a.nside > 8192;
-    const bool two = TB_FUSED_DPL_MAX > 1 && a.n_det > 32;
-    if (wide) return two ? launch_t<NEST, NNZ, HWP, DEBUG, true, TB_FUSED_DPL_MAX>(wl, a, sched, st)
-                         : launch_t<NEST, NNZ, HWP, DEBUG, true, 1>(wl, a, sched, st);
-    return two ? launch_t<NEST, NNZ, HWP, DEBUG, false, TB_FUSED_DPL_MAX>(wl, a, sched, st)
-               : launch_t<NEST, NNZ, HWP, DEBUG, false, 1>(wl, a, sched, st);
+    if (a.nside > kCompactMaxNside) return launch_t<NEST, NNZ, HWP, DEBUG, true, false>(wl, a, sched, st);
+    return launch_t<NEST, NNZ, HWP, DEBUG, false, false>(wl, a, sched, st);
 }
 
 // ============================================================================ few detectors
 // With fewer than kThinMaxDet detectors a 32-lane detector group leaves most lanes idle (C1: 4
 // detectors, 4 of 32 lanes).  Then THREAD = (chunk, detector): each thread builds its own
 // per-sample state from the boresight (consecutive threads share a chunk, so those loads are
-// L1 broadcasts) and runs the same per-det-sample arithmetic, run aggregation and flush as the
-// warp-per-item kernel (stage_a / stage_b / aggregate / flush), with the CTA's hit flags in
-// shared memory.
+// L1 broadcasts) and runs the same per-det-sample arithmetic, with a direct (per-thread) run
+// flush; the CTA's hit flags are gathered in its global2local cache.
 constexpr int kThinMaxDet = 8;
 
 template <bool NEST, int NNZ, bool HWP, bool WIDE>
 __global__ void __launch_bounds__(256) pointing_to_map_thin_kernel(const Chunk* __restrict__ chunks, int64_t n_chunks,
-                                                                  FusedArgs a, HealpixGeom g) {
+                                                                  FusedArgs a, HealpixGeom g, KeyConsts kc) {
     using P = typename PixT<WIDE>::T;
+    constexpr bool OFF = kOff<NNZ, P>;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    uint16_t* s_spread = reinterpret_cast<uint16_t*>(smem_raw);
-    uint8_t* s_hits = smem_raw + kSpreadBytes;
-    const CtaMem cm{s_spread, s_hits};
-    for (int i = threadIdx.x; i < 256; i += blockDim.x) {
-        unsigned v = 0u;
-        for (int b = 0; b < 8; ++b) v |= ((i >> b) & 1u) << (2 * b);
-        s_spread[i] = (uint16_t)v;
-    }
-    if (a.map.shared_hits)
-        for (int i = threadIdx.x; i < (int)a.map.n_submap; i += blockDim.x) s_hits[i] = 0;
+    uint16_t* s_g2l = reinterpret_cast<uint16_t*>(smem_raw);
+    __shared__ int s_nocache;
+    const MapGeom& mg = a.map;
+    if (threadIdx.x == 0) s_nocache = 0;
     __syncthreads();
+    if (mg.cache_g2l) {
+        for (int i = threadIdx.x; i < (int)mg.n_submap; i += blockDim.x) {
+            const int64_t v = __ldg(&mg.global2local[i]);
+            if (v >= (int64_t)kNoLoc) s_nocache = 1;
+            s_g2l[i] = v < 0 ? kNoLoc : (uint16_t)(v & 0x7fff);
+        }
+    }
+    __syncthreads();
+    const CtaMem cm{s_g2l, mg.cache_g2l && !s_nocache};
     const int64_t n_items = n_chunks * a.n_det;
     for (int64_t it = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; it < n_items;
          it += (int64_t)gridDim.x * blockDim.x) {
@@ -1184,46 +1077,72 @@ __global__ void __launch_bounds__(256) pointing_to_map_thin_kernel(const Chunk* 
         const Chunk ch = chunks[c];
         Slot<P> sl;
         load_slot<P>(sl, a, d, true, d);
+        auto flush = [&]() {
+            if (sl.run_key >= 0)
+                add_run<NNZ>(locate(key_to_pixel<NEST, OFF, WIDE>(sl.run_key, g), a, cm), sl.r0 * sl.sI,
+                             sl.r1 * sl.sQ, sl.r2 * sl.sU, a, d);
+        };
         for (int64_t s = ch.first; s < ch.first + ch.count; ++s) {
             if (a.shared_flags && (__ldg(&a.shared_flags[s]) & a.shared_flag_mask)) continue;  // no pixel (S2)
             const double2 q01 = __ldg(reinterpret_cast<const double2*>(a.boresight + 4 * s));
             const double2 q23 = __ldg(reinterpret_cast<const double2*>(a.boresight + 4 * s) + 1);
             double x[12];
             quat_to_matrix(q01.x, q01.y, q23.x, q23.y, x);
-            if (HWP && NNZ == 3) small_sincos(4.0 * __ldg(&a.hwp[s]), &x[10], &x[9]);
+            if (HWP && NNZ == 3) {
+                double s4, c4;
+                const double a4 = 4.0 * __ldg(&a.hwp[s]);
+                if (fabs(a4) < 1.6e6)
+                    small_sincos(a4, &s4, &c4);
+                else
+                    sincos(a4, &s4, &c4);
+                x[9] = c4;
+                x[10] = 2.0 * s4;
+                x[11] = 0.5 * s4;
+            }
             double tod = __ldg(&a.det_data[d * a.n_samp + s]);
             if (a.det_flags && (__ldg(&a.det_flags[d * a.n_samp + s]) & a.det_flag_mask)) tod = 0.0;
-            aggregate<NEST, NNZ, WIDE>(sl, a, g, cm);
-            det_sample<NEST, NNZ, HWP, false, WIDE>(sl, x, true, tod, g, a, d, s);
+            const StageA o = stage_a<NNZ, HWP, P>(sl, x, kc);
+            const P key = stage_b<NEST, NNZ, WIDE>(o, true, g, kc);
+            if (key != sl.run_key) {
+                flush();
+                sl.run_key = key;
+                sl.r0 = sl.r1 = sl.r2 = 0.0;
+            }
+            sl.r0 += tod;
+            if (NNZ == 3) {
+                const double t = tod * o.invr;
+                sl.r1 = fma(t, o.cw, sl.r1);
+                sl.r2 = fma(t, o.sw, sl.r2);
+            }
         }
-        aggregate<NEST, NNZ, WIDE>(sl, a, g, cm);
-        flush<NNZ, WIDE>(sl, a);
+        flush();
     }
-    if (a.map.shared_hits) {
+    if (a.hit_submaps && cm.cached) {
         __syncthreads();
-        for (int i = threadIdx.x; i < (int)a.map.n_submap; i += blockDim.x)
-            if (s_hits[i]) a.hit_submaps[i] = 1;
+        for (int i = threadIdx.x; i < (int)mg.n_submap; i += blockDim.x)
+            if (s_g2l[i] & kHitBit) a.hit_submaps[i] = 1;
     }
 }
 
 template <bool NEST, int NNZ, bool HWP>
 cudaError_t launch_thin(const WorkList& wl, const FusedArgs& a, cudaStream_t st) {
-    const size_t smem = kSpreadBytes + kSharedHitBytes;
+    const size_t smem = a.map.cache_g2l ? 2 * (size_t)a.map.n_submap : 0;
     const int64_t items = wl.n_chunks * a.n_det;
     const int64_t grid = std::min<int64_t>((items + 255) / 256, (int64_t)num_sms() * 8);
     t_fused_path = "thin (thread per chunk x detector, few detectors)";
-    if (a.nside > 8192)
-        pointing_to_map_thin_kernel<NEST, NNZ, HWP, true><<<(unsigned)grid, 256, smem, st>>>(wl.chunks, wl.n_chunks, a,
-                                                                                              make_geom(a.nside));
+    if (a.nside > kCompactMaxNside)
+        pointing_to_map_thin_kernel<NEST, NNZ, HWP, true><<<(unsigned)grid, 256, smem, st>>>(
+            wl.chunks, wl.n_chunks, a, make_geom(a.nside), make_key_consts(a.nside));
     else
-        pointing_to_map_thin_kernel<NEST, NNZ, HWP, false><<<(unsigned)grid, 256, smem, st>>>(wl.chunks, wl.n_chunks, a,
-                                                                                               make_geom(a.nside));
+        pointing_to_map_thin_kernel<NEST, NNZ, HWP, false><<<(unsigned)grid, 256, smem, st>>>(
+            wl.chunks, wl.n_chunks, a, make_geom(a.nside), make_key_consts(a.nside));
     return cudaGetLastError();
 }
 
 template <bool NEST, int NNZ, bool HWP>
 cudaError_t dispatch_debug(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
-    if (a.pixels_out || a.weights_out) return dispatch_shape<NEST, NNZ, HWP, true>(wl, a, sched, st);
+    // debug outputs and the dropped-sample counter run in the debug instantiation
+    if (a.pixels_out || a.weights_out || a.dropped) return dispatch_shape<NEST, NNZ, HWP, true>(wl, a, sched, st);
 #ifndef TB_NO_THIN
     if (a.n_det < kThinMaxDet) return launch_thin<NEST, NNZ, HWP>(wl, a, st);
 #endif
@@ -1240,33 +1159,35 @@ cudaError_t dispatch_hwp(const WorkList& wl, const FusedArgs& a, unsigned long l
 // toast_pointing_to_tod: pointing_to_map_kernel<..., SCAN = true>.
 template <bool NEST, int NNZ>
 cudaError_t dispatch_scan(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
-    const bool wide = a.nside > 8192;
+    const bool wide = a.nside > kCompactMaxNside;
     const bool hwp = a.hwp && NNZ == 3;
-    if (wide) return hwp ? launch_t<NEST, NNZ, true, false, true, 1, true>(wl, a, sched, st)
-                         : launch_t<NEST, NNZ, false, false, true, 1, true>(wl, a, sched, st);
-    return hwp ? launch_t<NEST, NNZ, true, false, false, 1, true>(wl, a, sched, st)
-               : launch_t<NEST, NNZ, false, false, false, 1, true>(wl, a, sched, st);
+    if (wide) return hwp ? launch_t<NEST, NNZ, true, false, true, true>(wl, a, sched, st)
+                         : launch_t<NEST, NNZ, false, false, true, true>(wl, a, sched, st);
+    return hwp ? launch_t<NEST, NNZ, true, false, false, true>(wl, a, sched, st)
+               : launch_t<NEST, NNZ, false, false, false, true>(wl, a, sched, st);
+}
+
+// Launch-side map geometry of the fused kernels: the submap count and whether the CTAs cache
+// global2local in shared memory.
+FusedArgs with_map_geom(FusedArgs a) {
+    MapGeom& m = a.map;
+    m.n_submap = (12 * a.nside * a.nside + m.n_pix_submap - 1) / m.n_pix_submap;
+    m.cache_g2l = m.n_submap <= kG2lCache;
+    return a;
 }
 
 }  // namespace
 
-cudaError_t launch_pointing_to_tod(const WorkList& wl, const FusedArgs& a, unsigned long long* sched,
+cudaError_t launch_pointing_to_tod(const WorkList& wl, const FusedArgs& a_in, unsigned long long* sched,
                                    cudaStream_t st) {
+    FusedArgs a = with_map_geom(a_in);
+    a.hit_submaps = nullptr;  // the scan marks nothing
     if (wl.n_chunks == 0 || a.n_det == 0) return cudaSuccess;
     if (a.nest) return a.nnz == 3 ? dispatch_scan<true, 3>(wl, a, sched, st) : dispatch_scan<true, 1>(wl, a, sched, st);
     return a.nnz == 3 ? dispatch_scan<false, 3>(wl, a, sched, st) : dispatch_scan<false, 1>(wl, a, sched, st);
 }
 
 const char* last_fused_path() { return t_fused_path; }
-
-// Launch-side map geometry of the fused kernel: the submap count and whether the hit flags
-// are gathered in shared memory.
-FusedArgs with_map_geom(FusedArgs a) {
-    MapGeom& m = a.map;
-    m.n_submap = (12 * a.nside * a.nside + m.n_pix_submap - 1) / m.n_pix_submap;
-    m.shared_hits = a.hit_submaps != nullptr && m.n_submap <= kSharedHitBytes;
-    return a;
-}
 
 cudaError_t launch_pointing_to_map(const WorkList& wl, const FusedArgs& a_in, unsigned long long* sched,
                                    cudaStream_t st) {

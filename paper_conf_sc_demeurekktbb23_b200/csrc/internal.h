@@ -35,16 +35,16 @@ struct MapGeom {
     const int64_t* global2local;
     int64_t n_pix_submap;
     int sm_shift;         // log2(n_pix_submap) if a power of two, else -1
-    // fused pointing_to_map only (set at launch): n_submap = 12 nside^2 / n_pix_submap, and
-    // whether the hit-submap flags are gathered in a per-CTA shared-memory copy (n_submap <=
-    // kSharedHitBytes) and written to hit_submaps once per CTA at the end.
+    // fused kernels only (set at launch): n_submap = 12 nside^2 / n_pix_submap, and whether each
+    // CTA caches global2local (as int16, with the hit flag in bit 15) in shared memory
+    // (n_submap <= kG2lCache); the hit flags then reach hit_submaps once per CTA, at its end.
     int64_t n_submap = 0;
-    int shared_hits = 0;
+    int cache_g2l = 0;
 };
 
-// Shared-memory hit-submap flags per CTA of the fused kernel (n_submap = 3072 at every nside
-// >= 16 with the 16x16-submap layout of the benchmarks).
-constexpr int kSharedHitBytes = 8192;
+// Shared-memory global2local cache of the fused kernels: up to kG2lCache submaps (3072 at every
+// nside >= 16 with the 16x16-submap layout of the benchmarks).
+constexpr int kG2lCache = 4096;
 
 struct FusedArgs {
     const double* fp_quats;
@@ -62,14 +62,20 @@ struct FusedArgs {
     int nest;
     int nnz;
     MapGeom map;
-    double* zmap;
+    double* zmap;          // fp64 map, or (map_f32) a float map at the same address
+    int map_f32;
     uint8_t* hit_submaps;
     int64_t* pixels_out;
     double* weights_out;
     int64_t n_det;
     int64_t n_samp;
+    // reading R3 (f4): per-detector polarisation angle [n_det] (NULL: 0) and the IAU sign of U
+    const double* gamma;
+    int iau;
+    // debug counter of det-samples whose hit submap has no storage (global2local < 0); NULL: off
+    unsigned long long* dropped;
     // pointing_to_tod (scan direction) only
-    const double* mapdata;
+    const double* mapdata;  // fp64 map, or (map_f32) a float map
     double data_scale;
     int should_zero;
     int should_subtract;
@@ -86,7 +92,7 @@ cudaError_t launch_pixels_healpix(const WorkList& wl, const int32_t* quat_index,
 cudaError_t launch_stokes_weights_iqu(const WorkList& wl, const int32_t* quat_index, const double* quats,
                                       const int32_t* weight_index, double* weights, const double* hwp,
                                       const double* epsilon, double cal, int64_t n_det, int64_t n_samp,
-                                      cudaStream_t st);
+                                      cudaStream_t st, const double* gamma = nullptr, int iau = 0);
 cudaError_t launch_build_noise_weighted(const WorkList& wl, const MapGeom& mg, double* zmap, int nnz,
                                         const int32_t* pixel_index, const int64_t* pixels,
                                         const int32_t* weight_index, const double* weights,

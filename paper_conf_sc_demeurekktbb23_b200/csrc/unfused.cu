@@ -148,12 +148,14 @@ template <bool HWP, bool IDX>
 __global__ void __launch_bounds__(kChunk, TB_A3_MINB) stokes_weights_kernel(
     const Chunk* __restrict__ chunks, int64_t n_chunks, const int32_t* __restrict__ quat_index,
     const double* __restrict__ quats, const int32_t* __restrict__ weight_index, double* __restrict__ weights,
-    const double* __restrict__ hwp, const double* __restrict__ epsilon, double cal, int64_t n_det, int64_t n_samp) {
+    const double* __restrict__ hwp, const double* __restrict__ epsilon, double cal, int64_t n_det, int64_t n_samp,
+    const double* __restrict__ gamma, int iau) {
     for (int64_t c = blockIdx.x; c < n_chunks; c += gridDim.x) {
         const Chunk ch = chunks[c];
         if ((int)threadIdx.x >= ch.count) continue;
         const int64_t s = ch.first + threadIdx.x;
         double c4 = 1.0, s4 = 0.0;
+        // reading R1: sincos of the exact 4 chi (full-range reduction) for any finite chi
         if (HWP) sincos(4.0 * __ldg(&hwp[s]), &s4, &c4);
         FOR_DET_TILES(d0) {
             double q[kDT][4];
@@ -175,11 +177,18 @@ __global__ void __launch_bounds__(kChunk, TB_A3_MINB) stokes_weights_kernel(
                 if (HWP) {
                     cq = c2 * c4 - s2 * s4;
                     sq = s2 * c4 + c2 * s4;
+                    if (gamma) {  // reading R3: rotate by -4 gamma (a variant; one sincos per det-sample)
+                        double sg, cg;
+                        sincos(4.0 * __ldg(&gamma[d]), &sg, &cg);
+                        const double q = fma(cg, cq, sg * sq), u = fma(cg, sq, -sg * cq);
+                        cq = q;
+                        sq = u;
+                    }
                 }
                 double* out = weights + (row_of<IDX>(weight_index, d) * n_samp + s) * 3;
                 out[0] = cal;
                 out[1] = etacal * cq;
-                out[2] = etacal * sq;
+                out[2] = iau ? -(etacal * sq) : etacal * sq;
             }
         }
     }
@@ -323,14 +332,16 @@ cudaError_t launch_pixels_healpix(const WorkList& wl, const int32_t* quat_index,
 cudaError_t launch_stokes_weights_iqu(const WorkList& wl, const int32_t* quat_index, const double* quats,
                                       const int32_t* weight_index, double* weights, const double* hwp,
                                       const double* epsilon, double cal, int64_t n_det, int64_t n_samp,
-                                      cudaStream_t st) {
+                                      cudaStream_t st, const double* gamma, int iau) {
     if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
     if (hwp)
         (quat_index || weight_index ? stokes_weights_kernel<true, true> : stokes_weights_kernel<true, false>)<<<grid_for(wl, n_det), kChunk, 0, st>>>(
-            wl.chunks, wl.n_chunks, quat_index, quats, weight_index, weights, hwp, epsilon, cal, n_det, n_samp);
+            wl.chunks, wl.n_chunks, quat_index, quats, weight_index, weights, hwp, epsilon, cal, n_det, n_samp, gamma,
+            iau);
     else
         (quat_index || weight_index ? stokes_weights_kernel<false, true> : stokes_weights_kernel<false, false>)<<<grid_for(wl, n_det), kChunk, 0, st>>>(
-            wl.chunks, wl.n_chunks, quat_index, quats, weight_index, weights, hwp, epsilon, cal, n_det, n_samp);
+            wl.chunks, wl.n_chunks, quat_index, quats, weight_index, weights, hwp, epsilon, cal, n_det, n_samp, gamma,
+            iau);
     return cudaGetLastError();
 }
 

@@ -62,14 +62,15 @@ class DeviceWorkload:
             intervals=binding.intervals_host(w.intervals),
         )
 
-    def pointing_to_map(self, zmap=None, hit_submaps=None, pixels_out=None, weights_out=None, stream=None):
+    def pointing_to_map(self, zmap=None, hit_submaps=None, pixels_out=None, weights_out=None, stream=None,
+                        gamma=None, iau=False, dropped=None):
         w = self.w
         return binding.pointing_to_map(
             self.fp_quats, self.boresight, self.epsilon, w.cal, self.det_scale, self.det_data, self.intervals,
             w.nside, w.nest, w.nnz, self.global2local, w.n_pix_submap, self.zmap if zmap is None else zmap,
             hwp=self.hwp, det_flags=self.det_flags, det_flag_mask=w.det_flag_mask, shared_flags=self.shared_flags,
             shared_flag_mask=w.shared_flag_mask, hit_submaps=self.hit_submaps if hit_submaps is None else hit_submaps,
-            pixels_out=pixels_out, weights_out=weights_out, stream=stream)
+            pixels_out=pixels_out, weights_out=weights_out, stream=stream, gamma=gamma, iau=iau, dropped=dropped)
 
     def raw_args(self, stream=None, zmap=None, det_data=None):
         """Pre-marshalled argument tuple of toast_pointing_to_map (no per-call Python checks)."""

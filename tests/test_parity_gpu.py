@@ -41,9 +41,10 @@ def _sin_theta(quats):
     return 2.0 * np.sqrt(np.clip(a * (1.0 - a), 0, None))
 
 
-def _oracle_fused(w):
+def _oracle_fused(w, gamma=None, iau=False):
     zmap = np.zeros((w.n_submap, w.n_pix_submap, w.nnz))
     absmap = np.zeros_like(zmap)
+    t2map = np.zeros_like(zmap)
     hits = np.zeros(w.n_submap, np.uint8)
     pix = np.full((w.n_det, w.n_samp), -7, np.int64)
     wts = np.zeros((w.n_det, w.n_samp, w.nnz))
@@ -51,17 +52,37 @@ def _oracle_fused(w):
                            w.nest, w.nnz, w.global2local, w.n_pix_submap, zmap=zmap, hwp=w.hwp, det_flags=w.det_flags,
                            det_flag_mask=w.det_flag_mask, shared_flags=w.shared_flags,
                            shared_flag_mask=w.shared_flag_mask, hit_submaps=hits, pixels_out=pix, weights_out=wts,
-                           absmap=absmap)
-    return zmap, absmap, hits, pix, wts
+                           absmap=absmap, gamma=gamma, iau=iau, t2map=t2map)
+    return zmap, absmap, hits, pix, wts, t2map
 
 
-def _probe(w):
+def _probe(w, gamma=None, iau=False):
     def probe(d, s):
         flagged = w.shared_flags is not None and bool(w.shared_flags[s] & w.shared_flag_mask)
-        _, _, v = oracle.det_sample_probe(w.fp_quats[d], w.boresight[s], 0.0 if w.hwp is None else w.hwp[s],
-                                          w.epsilon[d], w.cal, flagged, w.nside, w.nest)
+        _, _, v = oracle.det_sample_probe(w.fp_quats[d], w.boresight[s], None if w.hwp is None else w.hwp[s],
+                                          w.epsilon[d], w.cal, flagged, w.nside, w.nest,
+                                          gamma=0.0 if gamma is None else gamma[d], iau=iau)
         return v
     return probe
+
+
+def _sin_theta_of(w):
+    probe = _probe(w)
+
+    def sth(d, s):
+        v = probe(d, s)
+        return float(np.hypot(v[0], v[1]))
+    return sth
+
+
+def _check_fused_map(gpu_map, ref, mism, pg, w):
+    """T4 of a fused map against the oracle's, the near-boundary decisions reconciled."""
+    zo, absmap, _, po, wo, t2map = ref
+    zo_r, abs_r = zo.copy(), absmap.copy()
+    t2_r = t2map.copy()
+    reconcile_map(zo_r, abs_r, mism, pg, po, wo, w, w.global2local, w.n_pix_submap, t2map=t2_r,
+                  sin_theta=_sin_theta_of(w))
+    check_map(gpu_map, zo_r, abs_r, t2_r)
 
 
 FUSED_CASES = {
@@ -80,7 +101,8 @@ FUSED_CASES = {
 @pytest.mark.parametrize("case", list(FUSED_CASES))
 def test_fused_pointing_to_map(case):
     w = synth.make_workload(**FUSED_CASES[case])
-    zo, absmap, ho, po, wo = _oracle_fused(w)
+    ref = _oracle_fused(w)
+    zo, absmap, ho, po, wo, t2map = ref
     dw = DeviceWorkload.upload(w, DEV)
     n_in = int(_in_mask(w.intervals, 1, w.n_samp).sum()) * w.n_det
 
@@ -95,8 +117,7 @@ def test_fused_pointing_to_map(case):
     eta_cal = (1 - w.epsilon) / (1 + w.epsilon) * w.cal
     mask = np.array(_in_mask(w.intervals, w.n_det, w.n_samp))
     check_weights(wg, wo, _sin_theta(quats), eta_cal, w.cal, mask)
-    zo_r, abs_r = reconcile_map(zo.copy(), absmap.copy(), mism, pg, po, wo, w, w.global2local, w.n_pix_submap)
-    check_map(dw.zmap.cpu().numpy(), zo_r, abs_r)
+    _check_fused_map(dw.zmap.cpu().numpy(), ref, mism, pg, w)
     hits_expect = np.zeros(w.n_submap, np.uint8)
     good = pg[pg >= 0]
     hits_expect[np.unique(good // w.n_pix_submap)] = 1
@@ -109,7 +130,7 @@ def test_fused_pointing_to_map(case):
     dw.hit_submaps.zero_()
     dw.pointing_to_map()
     torch.cuda.synchronize()
-    check_map(dw.zmap.cpu().numpy(), zo_r, abs_r)
+    _check_fused_map(dw.zmap.cpu().numpy(), ref, mism, pg, w)
     np.testing.assert_array_equal(dw.hit_submaps.cpu().numpy(), hits_expect)
 
 
@@ -117,7 +138,8 @@ def test_fused_tma_and_cp_async_paths():
     """The same workload staged by TMA (aligned TOD) and by cp.async (TOD base only 8-byte
     aligned, so the TMA constraints fail) gives the oracle's map either way."""
     w = synth.make_workload("c2", n_det=36, n_samp=64_000)
-    zo, absmap, ho, po, wo = _oracle_fused(w)
+    ref = _oracle_fused(w)
+    po = ref[3]
     buf = torch.empty(w.n_det * w.n_samp + 1, dtype=torch.float64, device=DEV)
     odd = buf[1:].view(w.n_det, w.n_samp)
     odd.copy_(torch.from_numpy(np.ascontiguousarray(w.det_data)))
@@ -131,8 +153,13 @@ def test_fused_tma_and_cp_async_paths():
         pg = pix_g.cpu().numpy()
         n_in = int(_in_mask(w.intervals, 1, w.n_samp).sum()) * w.n_det
         mism = classify_pixel_mismatches(pg, po, _probe(w), w.nside, w.nest, n_in)
-        zo_r, abs_r = reconcile_map(zo.copy(), absmap.copy(), mism, pg, po, wo, w, w.global2local, w.n_pix_submap)
-        check_map(dw.zmap.cpu().numpy(), zo_r, abs_r)
+        _check_fused_map(dw.zmap.cpu().numpy(), ref, mism, pg, w)
+        # production instantiation on the same staging path
+        dw.zmap.zero_()
+        dw.pointing_to_map()
+        torch.cuda.synchronize()
+        assert binding.last_fused_path().startswith(path), binding.last_fused_path()
+        _check_fused_map(dw.zmap.cpu().numpy(), ref, mism, pg, w)
 
 
 def test_fused_integer_inputs_give_exact_hit_counts():
@@ -141,7 +168,7 @@ def test_fused_integer_inputs_give_exact_hit_counts():
     w = synth.make_workload("c2", n_det=20, n_samp=150_000, nnz=1)
     w.det_data = np.ones_like(w.det_data)
     w.det_scale = np.ones_like(w.det_scale)
-    zo, absmap, ho, po, wo = _oracle_fused(w)
+    zo, absmap, ho, po, wo, _ = _oracle_fused(w)
     dw = DeviceWorkload.upload(w, DEV)
     pix_g = torch.full((w.n_det, w.n_samp), -7, dtype=torch.int64, device=DEV)
     dw.pointing_to_map(pixels_out=pix_g)
@@ -173,14 +200,13 @@ def test_fused_extreme_nside(nside, nest):
         np.testing.assert_array_equal(dw.hit_submaps.cpu().numpy(), hits)
         assert np.all(dw.zmap.cpu().numpy() == 0)
         return
-    zo, absmap, ho, po, wo = _oracle_fused(w)
-    dw.zmap = torch.zeros(zo.shape, dtype=torch.float64, device=DEV)
+    ref = _oracle_fused(w)
+    dw.zmap = torch.zeros(ref[0].shape, dtype=torch.float64, device=DEV)
     dw.hit_submaps = torch.zeros(w.n_submap, dtype=torch.uint8, device=DEV)
     dw.pointing_to_map(pixels_out=pix_g)
     pg = pix_g.cpu().numpy()
-    mism = classify_pixel_mismatches(pg, po, _probe(w), nside, nest, n_in)
-    zo_r, abs_r = reconcile_map(zo, absmap, mism, pg, po, wo, w, w.global2local, w.n_pix_submap)
-    check_map(dw.zmap.cpu().numpy(), zo_r, abs_r)
+    mism = classify_pixel_mismatches(pg, ref[3], _probe(w), nside, nest, n_in)
+    _check_fused_map(dw.zmap.cpu().numpy(), ref, mism, pg, w)
 
 
 @pytest.mark.parametrize("name,n_det", [("c1", 4), ("c2", 40)])  # thread path and warp path
@@ -201,14 +227,14 @@ def test_fused_production_wide_and_many_submaps(name, n_det):
     # nside 64 with 4-pixel submaps: 12288 submaps
     w = synth.make_workload(name, n_det=n_det, n_samp=20_000, nside=64)
     w.n_pix_submap = 4
-    zo, absmap, ho, po, wo = _oracle_fused(w)
+    zo, absmap, ho, po, wo, t2map = _oracle_fused(w)
     dw = DeviceWorkload.upload(w, DEV, alloc_map=False)
     dw.zmap = torch.zeros(zo.shape, dtype=torch.float64, device=DEV)
     dw.hit_submaps = torch.zeros(w.n_submap, dtype=torch.uint8, device=DEV)
     assert w.n_submap > 8192
     dw.pointing_to_map()
     torch.cuda.synchronize()
-    check_map(dw.zmap.cpu().numpy(), zo, absmap)
+    check_map(dw.zmap.cpu().numpy(), zo, absmap, t2map)
     np.testing.assert_array_equal(dw.hit_submaps.cpu().numpy(), ho)
 
 
@@ -221,12 +247,12 @@ def test_fused_edge_intervals(n_samp):
     for ivs in ([], [(0, 0)], [(0, 254), (300, 555), (600, 856), (last, last)], [(10, 10), (11, 11), (12, 4000)],
                 [(1, 1), (3, 17), (33, 160), (161, 290), (4001, last)], [(last - 16, last)]):
         w.intervals = ivs
-        zo, absmap, ho, po, wo = _oracle_fused(w)
+        zo, absmap, ho, po, wo, t2map = _oracle_fused(w)
         dw = DeviceWorkload.upload(w, DEV)
         pix_g = torch.full((w.n_det, w.n_samp), -7, dtype=torch.int64, device=DEV)
         dw.pointing_to_map(pixels_out=pix_g)
         np.testing.assert_array_equal(pix_g.cpu().numpy(), po)  # includes untouched -7 outside intervals
-        check_map(dw.zmap.cpu().numpy(), zo, absmap)
+        check_map(dw.zmap.cpu().numpy(), zo, absmap, t2map)
         np.testing.assert_array_equal(dw.hit_submaps.cpu().numpy(), ho)
 
 
@@ -234,13 +260,13 @@ def test_fused_global2local_permuted():
     w = synth.make_workload("c1", n_samp=30_000)
     rng = np.random.default_rng(3)
     perm = rng.permutation(w.n_submap).astype(np.int64)
-    zo = np.zeros((w.n_submap, w.n_pix_submap, 3)); absmap = np.zeros_like(zo)
+    zo = np.zeros((w.n_submap, w.n_pix_submap, 3)); absmap = np.zeros_like(zo); t2map = np.zeros_like(zo)
     oracle.pointing_to_map(w.fp_quats, w.boresight, w.epsilon, w.cal, w.det_scale, w.det_data, w.intervals, w.nside,
-                           w.nest, 3, perm, w.n_pix_submap, zmap=zo, absmap=absmap)
+                           w.nest, 3, perm, w.n_pix_submap, zmap=zo, absmap=absmap, t2map=t2map)
     dw = DeviceWorkload.upload(w, DEV)
     dw.global2local = torch.from_numpy(perm).to(DEV)
     dw.pointing_to_map()
-    check_map(dw.zmap.cpu().numpy(), zo, absmap)
+    check_map(dw.zmap.cpu().numpy(), zo, absmap, t2map)
 
 
 def test_fused_compact_map_domain():
@@ -249,7 +275,7 @@ def test_fused_compact_map_domain():
     map on every hit submap (bench.py --reduce scatter runs exactly this)."""
     from paper_conf_sc_demeurekktbb23_b200 import dist as tdist
     w = synth.make_workload("c5", n_det=40, n_samp=40_000)
-    zo, absmap, ho, po, wo = _oracle_fused(w)
+    zo, absmap, ho, po, wo, t2map = _oracle_fused(w)
     dw = DeviceWorkload.upload(w, DEV)
     dw.pointing_to_map()
     g2l, n_hit = tdist.compact_global2local(dw.hit_submaps)
@@ -262,9 +288,9 @@ def test_fused_compact_map_domain():
     torch.cuda.synchronize()
     hit = np.nonzero(ho)[0]
     np.testing.assert_array_equal(np.nonzero(dw.hit_submaps.cpu().numpy())[0], hit)
-    check_map(zc[:n_hit].cpu().numpy(), zo[hit], absmap[hit])
+    check_map(zc[:n_hit].cpu().numpy(), zo[hit], absmap[hit], t2map[hit])
     full = tdist.gather_map(zc[:own.per_rank], own, g2l, w.n_submap)
-    check_map(full.cpu().numpy(), zo, absmap)
+    check_map(full.cpu().numpy(), zo, absmap, t2map)
 
 
 @pytest.mark.parametrize("dets", [(0, 0), (5, 6), (0, 7), (0, 8), (0, 33)])
@@ -272,11 +298,11 @@ def test_fused_detector_counts(dets):
     """No detector (a no-op), one and seven detectors (the thread-per-(chunk, detector) path), eight
     (the warp path with 24 idle lanes), one full warp group plus a one-detector group."""
     w = synth.make_workload("c2", n_det=64, n_samp=30_000, det_range=dets)
-    zo, absmap, ho, po, wo = _oracle_fused(w)
+    zo, absmap, ho, po, wo, t2map = _oracle_fused(w)
     dw = DeviceWorkload.upload(w, DEV)
     dw.pointing_to_map()
     torch.cuda.synchronize()
-    check_map(dw.zmap.cpu().numpy(), zo, absmap)
+    check_map(dw.zmap.cpu().numpy(), zo, absmap, t2map)
     np.testing.assert_array_equal(dw.hit_submaps.cpu().numpy(), ho)
 
 
@@ -440,7 +466,9 @@ def test_scan_map(chain, zero, subtract):
 
 def test_round_trip_scan_then_accumulate():
     """C3-shaped round trip on the GPU chain (A1 -> A2 -> A3 -> A5 -> A4) vs the oracle chain;
-    smooth map I = cos 3theta, Q = sin 2phi sin theta, U = cos phi sin theta."""
+    smooth map I = cos 3theta, Q = sin 2phi sin theta, U = cos phi sin theta.  Near-boundary
+    pixel decisions (rule T1) are reconciled: the oracle chain is re-run with the GPU's pixel at
+    exactly the samples the oracle classifier proves to lie within 1e-12 rad of a boundary."""
     w = synth.make_workload("c3", n_det=20, n_samp=30_000, nside=256)
     from independent import ring_centres
     z, ph = ring_centres(w.nside)
@@ -448,22 +476,12 @@ def test_round_trip_scan_then_accumulate():
     th = np.arccos(z)
     m_ring = np.stack([np.cos(3 * th), np.sin(2 * ph) * st, np.cos(ph) * st], -1)
     m = m_ring.reshape(w.n_submap, w.n_pix_submap, 3)  # RING ordering, identity global2local
-    # oracle chain
-    quats = oracle.pointing_detector(w.fp_quats, w.boresight, w.intervals, w.shared_flags, w.shared_flag_mask)
-    pix, _ = oracle.pixels_healpix(quats, w.intervals, w.nside, w.nest, w.n_pix_submap, w.shared_flags,
-                                   w.shared_flag_mask)
-    wts = oracle.stokes_weights_iqu(quats, w.intervals, w.epsilon, w.cal)
-    tod = np.zeros((w.n_det, w.n_samp))
-    oracle.scan_map(m, w.global2local, w.n_pix_submap, pix, wts, tod, w.intervals)
-    ref = np.zeros_like(m); absmap = np.zeros_like(m)
-    oracle.build_noise_weighted(ref, w.global2local, w.n_pix_submap, pix, wts, tod, w.det_scale, w.intervals,
-                                shared_flags=w.shared_flags, shared_flag_mask=w.shared_flag_mask, absmap=absmap)
     # GPU chain
     qg = torch.zeros((w.n_det, w.n_samp, 4), dtype=torch.float64, device=DEV)
     sf = _cuda(w.shared_flags, torch.uint8)
     binding.pointing_detector(_cuda(w.fp_quats, torch.float64), _cuda(w.boresight, torch.float64), w.intervals, qg,
                               shared_flags=sf, shared_flag_mask=w.shared_flag_mask)
-    pg = torch.full((w.n_det, w.n_samp), -1, dtype=torch.int64, device=DEV)
+    pg = torch.full((w.n_det, w.n_samp), -7, dtype=torch.int64, device=DEV)  # -7: untouched, as the oracle's
     binding.pixels_healpix(qg, w.intervals, w.nside, w.nest, w.n_pix_submap, pg, shared_flags=sf,
                            shared_flag_mask=w.shared_flag_mask)
     wg = torch.zeros((w.n_det, w.n_samp, 3), dtype=torch.float64, device=DEV)
@@ -474,11 +492,41 @@ def test_round_trip_scan_then_accumulate():
     zg = torch.zeros(m.shape, dtype=torch.float64, device=DEV)
     binding.build_noise_weighted(zg, g2l, w.n_pix_submap, pg, wg, tg, _cuda(w.det_scale, torch.float64), w.intervals,
                                  shared_flags=sf, shared_flag_mask=w.shared_flag_mask)
+    # oracle chain
+    quats = oracle.pointing_detector(w.fp_quats, w.boresight, w.intervals, w.shared_flags, w.shared_flag_mask)
+    pix, _ = oracle.pixels_healpix(quats, w.intervals, w.nside, w.nest, w.n_pix_submap, w.shared_flags,
+                                   w.shared_flag_mask)
+    wts = oracle.stokes_weights_iqu(quats, w.intervals, w.epsilon, w.cal)
     pgn = pg.cpu().numpy()
-    if not np.array_equal(pgn, pix):
-        pytest.skip("near-boundary pixel mismatch; covered by the pixel tests")
-    np.testing.assert_allclose(tg.cpu().numpy(), tod, rtol=0, atol=1e-12 * 3)
-    check_map(zg.cpu().numpy(), ref, absmap + 1e-2 * np.abs(ref))  # tod carries the T3 error into the map
+    n_in = int(_in_mask(w.intervals, 1, w.n_samp).sum()) * w.n_det
+    mism = classify_pixel_mismatches(pgn, pix, lambda d, s: oracle.quat_rotate(quats[d, s], [0, 0, 1.0]), w.nside,
+                                     w.nest, n_in)
+    pix_r = pix.copy()
+    pix_r[mism] = pgn[mism]  # admissible decisions (T1), proven near a boundary above
+    tod = np.zeros((w.n_det, w.n_samp)); bsc = np.zeros_like(tod)
+    oracle.scan_map(m, w.global2local, w.n_pix_submap, pix_r, wts, tod, w.intervals, bscale=bsc)
+    ref = np.zeros_like(m); absmap = np.zeros_like(m)
+    oracle.build_noise_weighted(ref, w.global2local, w.n_pix_submap, pix_r, wts, tod, w.det_scale, w.intervals,
+                                shared_flags=w.shared_flags, shared_flag_mask=w.shared_flag_mask, absmap=absmap)
+    # T3 on the timestream: 1e-12 B + the T2 weight tolerance carried by |m_Q|, |m_U| (<= 1)
+    sth = _sin_theta(quats)
+    eta_cal = (1 - w.epsilon) / (1 + w.epsilon) * w.cal
+    t2 = np.abs(eta_cal)[:, None] * np.maximum(1e-12, 1e-15 / np.maximum(sth, 1e-300))
+    tol_tod = 1e-12 * bsc + 2 * t2 + 4e-16 * np.abs(tod)
+    got = tg.cpu().numpy()
+    assert np.all(np.abs(got - tod) <= tol_tod)
+    # T4 on the map, plus what the tolerated tod and weight differences carry into it
+    good = (pix_r >= 0) & np.array(_in_mask(w.intervals, w.n_det, w.n_samp))
+    d_idx = np.nonzero(good)
+    flat = pix_r[good]
+    extra = np.zeros((m.shape[0] * m.shape[1], 3))
+    scale = w.det_scale[d_idx[0]]
+    for k in range(3):
+        e = scale * tol_tod[good] * np.abs(wts[..., k][good])
+        if k > 0:
+            e = e + scale * np.abs(tod[good]) * t2[good]
+        np.add.at(extra[:, k], flat, e)
+    check_map(zg.cpu().numpy(), ref, absmap, extra=extra.reshape(m.shape))
 
 
 def test_invalid_arguments_are_rejected():
