@@ -23,7 +23,7 @@ def sources():
 
 def _deps():
     return sources() + sorted(glob.glob(os.path.join(CSRC, "*.cuh"))) + sorted(glob.glob(os.path.join(CSRC, "*.h"))) \
-        + [os.path.join(INCLUDE, "toast_b200.h")]
+        + sorted(glob.glob(os.path.join(INCLUDE, "*.h")))
 
 
 def up_to_date() -> bool:

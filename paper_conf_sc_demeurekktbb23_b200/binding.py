@@ -74,6 +74,7 @@ def load():
     L.toast_template_offset_add_to_signal.argtypes = [I64, P, P, P, P, P, I64, I64, I64, P]
     L.toast_template_offset_project_signal.argtypes = [I64, P, P, P, P, P, P, U8, P, I64, I64, I64, P]
     L.toast_template_offset_apply_diag_precond.argtypes = [P, P, P, I64, P]
+    L.toast_synth_tod.argtypes = [P, P, P, I64, I64, ctypes.c_uint64, ctypes.c_uint64, P]
     for name in EXPORTED[4:]:
         getattr(L, name).restype = I32
     _lib = L
@@ -85,7 +86,7 @@ EXPORTED = ("toast_last_error", "toast_version", "toast_last_fused_path", "toast
             "toast_build_noise_weighted", "toast_scan_map", "toast_pointing_to_map", "toast_pointing_to_map_ex",
             "toast_pointing_to_tod", "toast_pointing_to_tod_ex", "toast_stokes_weights_i", "toast_noise_weight",
             "toast_template_offset_add_to_signal", "toast_template_offset_project_signal",
-            "toast_template_offset_apply_diag_precond")
+            "toast_template_offset_apply_diag_precond", "toast_synth_tod")
 
 
 def version() -> str:
@@ -410,6 +411,17 @@ def template_offset_apply_diag_precond(offset_var, amp_in, amp_out, stream=None)
           c(amp_in, torch.float64, "amp_in", shape=(n,)), c(amp_out, torch.float64, "amp_out", shape=(n,)), n,
           stream=stream)
     return amp_out
+
+
+def synth_tod(out, sigma, det_ids, seed: int, stream_id: int = 1, stream=None):
+    """The seeded synthetic timestream on the device (include/toast_b200_synth.h): a bench / test
+    INPUT generator, bit-identical to synth.tod_rows; none of the method's arithmetic."""
+    c = _Call("toast_synth_tod")
+    n_det, n_samp = out.shape
+    c.run(load().toast_synth_tod, c(out, torch.float64, "out", shape=(n_det, n_samp)),
+          c(sigma, torch.float64, "sigma", shape=(n_det,)), c(det_ids, torch.int64, "det_ids", shape=(n_det,)),
+          n_det, n_samp, int(seed) & ((1 << 64) - 1), int(stream_id), stream=stream)
+    return out
 
 
 def pointing_to_map_raw(args: tuple):
