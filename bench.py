@@ -303,22 +303,11 @@ def main():
     binding.load()
     name = args.workload
     shard = args.shard if args.shard != "auto" else ("det" if name in ("c4", "c5m") else "obs")
-    if name == "c5m":
-        shard = "det" if world > 1 else "obs"
 
-    # ---- this rank's work: a list of (observation, detector range) units
+    # ---- this rank's work: (observation, detector range) units (dist.work_plan)
     from paper_conf_sc_demeurekktbb23_b200 import synth
     full_det = synth.CONFIGS[base_name(name)][1]
-    if name == "c5m":
-        # LPT over (observation, 256-detector block) units; whole observations on one GPU
-        units = tdist.make_units(C5M_OBS, full_det, [1] * C5M_OBS, 256 if world > 1 else full_det)
-        mine = tdist.plan_shards(units, world)[rank]
-        work = [(u.obs, (u.d0, u.d1) if world > 1 else None) for u in mine]
-    elif shard == "det" and world > 1:
-        per = (full_det + world - 1) // world
-        work = [(0, (rank * per, min(full_det, (rank + 1) * per)))]
-    else:
-        work = [(rank, None)]
+    work = tdist.work_plan(C5M_OBS if name == "c5m" else 1, full_det, world, rank, shard)
     obs = [Obs(name, o, dr, dev) for o, dr in work]
     w0 = obs[0].w
     n_submap, nps, nnz = w0.n_submap, w0.n_pix_submap, w0.nnz

@@ -63,6 +63,26 @@ def plan_shards(units: Sequence[Unit], world: int) -> List[List[Unit]]:
     return out
 
 
+def work_plan(n_obs: int, n_det: int, world: int, rank: int, shard: str, det_block: int = 256,
+              first_obs: int = 0) -> List[Tuple[int, Optional[Tuple[int, int]]]]:
+    """This rank's work as (observation, detector range or None = all) pairs — the plan bench.py
+    runs:
+      shard="det": one observation (n_obs = 1) cut into `world` contiguous detector blocks
+                   (C4: 2048 / 8 = 256 detectors per GPU), or several observations cut into
+                   `det_block` blocks and LPT-balanced (C5m); strong scaling;
+      shard="obs": observation first_obs + rank on every rank (weak scaling)."""
+    if shard == "obs":
+        return [(first_obs + rank, None)]
+    if world == 1:
+        return [(first_obs + o, None) for o in range(n_obs)]
+    if n_obs == 1:
+        per = -(-n_det // world)
+        lo, hi = min(n_det, rank * per), min(n_det, (rank + 1) * per)
+        return [(first_obs, (lo, hi))] if hi > lo else []
+    units = make_units(n_obs, n_det, [1] * n_obs, det_block)
+    return [(first_obs + u.obs, (u.d0, u.d1)) for u in plan_shards(units, world)[rank]]
+
+
 def union_hit_submaps(hit_submaps: torch.Tensor, group=None) -> torch.Tensor:
     """In-place all_reduce(MAX) of the per-rank hit-submap flags (uint8, n_submap)."""
     if dist.is_initialized() and dist.get_world_size(group) > 1:

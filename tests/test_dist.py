@@ -158,3 +158,62 @@ def test_two_rank_sparse_map_domain_reduce_scatter():
         # the owned block holds exactly this rank's slice of the hit submaps, fully summed
         check_map(block[:hi - lo], zref[hit_idx[lo:hi]], absmap[hit_idx[lo:hi]])
     assert res[0][5] == res[1][4]  # the two blocks tile the hit submaps
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 8])
+def test_work_plan_covers_every_detector_once(world):
+    """bench.py's sharding (dist.work_plan): the ranks' detector ranges partition the focal plane
+    (one observation, C4 style) / the (observation, block) units (several, C5m style)."""
+    for n_obs in (1, 18):
+        seen = []
+        for r in range(world):
+            for o, dr in tdist.work_plan(n_obs, 2048, world, r, "det"):
+                lo, hi = dr if dr is not None else (0, 2048)
+                seen += [(o, d) for d in range(lo, hi)]
+        assert sorted(seen) == [(o, d) for o in range(n_obs) for d in range(2048)]
+    assert [tdist.work_plan(1, 64, world, r, "obs") for r in range(world)] == [[(r, None)] for r in range(world)]
+
+
+def _bench_plan_worker(rank, world, port, q):
+    """Each rank runs THE bench's plan (dist.work_plan) on a C4-shaped detector split, accumulates
+    its units with the oracle, and the packed reduction sums them."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import oracle
+    from paper_conf_sc_demeurekktbb23_b200 import synth
+    n_det, n_samp = 12, 6000
+    base = synth.make_workload("c4", n_det=n_det, n_samp=n_samp, nside=64)
+    z = np.zeros((base.n_submap, base.n_pix_submap, 3))
+    hits = np.zeros(base.n_submap, np.uint8)
+    for o, dr in tdist.work_plan(1, n_det, world, rank, "det"):
+        w = synth.make_workload("c4", n_det=n_det, n_samp=n_samp, nside=64, obs=o, det_range=dr)
+        oracle.pointing_to_map(w.fp_quats, w.boresight, w.epsilon, w.cal, w.det_scale, w.det_data, w.intervals,
+                               w.nside, w.nest, 3, w.global2local, w.n_pix_submap, zmap=z, hit_submaps=hits)
+    zt, ht = torch.from_numpy(z), torch.from_numpy(hits)
+    tdist.union_hit_submaps(ht)
+    tdist.reduce_map(zt, hit_submaps=ht)
+    if rank == 0:
+        q.put(zt.numpy().copy())
+    dist.barrier()
+
+
+def test_bench_work_plan_reduced_equals_full_oracle_map():
+    import oracle
+    from paper_conf_sc_demeurekktbb23_b200 import synth
+    from parity import check_map
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_bench_plan_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    zsum = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    w = synth.make_workload("c4", n_det=12, n_samp=6000, nside=64)
+    zref = np.zeros_like(zsum); absmap = np.zeros_like(zsum)
+    oracle.pointing_to_map(w.fp_quats, w.boresight, w.epsilon, w.cal, w.det_scale, w.det_data, w.intervals, w.nside,
+                           w.nest, 3, w.global2local, w.n_pix_submap, zmap=zref, absmap=absmap)
+    check_map(zsum, zref, absmap)
