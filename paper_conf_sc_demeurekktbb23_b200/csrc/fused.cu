@@ -142,6 +142,15 @@ struct alignas(128) SflgSlot {
     unsigned long long mbar;
     uint8_t pad[104];
 };
+// A finished run waiting in the warp's flush queue (QUEUE kernels): its compact key, the lane
+// (detector) that produced it and its scaled sums.
+struct alignas(16) QEntry {
+    int key;
+    int src;
+    double r0, r1, r2;
+};
+constexpr int kQ = 32;  // queue entries per warp
+
 struct alignas(1024) WarpSmem {
     double tod[2][32][16];  // 1024-aligned (the 128-byte swizzle pattern spans 1 KB)
     uint8_t flg[2][32][16];
@@ -149,8 +158,9 @@ struct alignas(1024) WarpSmem {
     double hwp[2][16];
     SflgSlot sf[2];
     double st[16][12];      // per-sample state: B[0..8], c4, 2 s4, s4 / 2
+    QEntry q[kQ];           // the flush queue (QUEUE kernels)
 };
-static_assert(sizeof(WarpSmem) == 12288, "12 KB per warp");
+static_assert(sizeof(WarpSmem) == 13312, "13 KB per warp");
 
 // Pixel index / key type: 32-bit compact keys up to nside 4096, else the 64-bit pixel itself.
 template <bool WIDE>
@@ -466,7 +476,10 @@ template <bool NEST, int NNZ, bool OFF>
 __device__ __forceinline__ void flush_lean(int key, double r0, double r1, double r2, const FusedArgs& a,
                                            const HealpixGeom& g, uint16_t* g2l) {
     const MapGeom& mg = a.map;
-    const unsigned pix = (unsigned)ckey_to_pix_bf<NEST, OFF>(key, g);
+    // branchy decode: the lanes of a warp (a 5-degree focal plane) are almost always all in the
+    // belt or all in a cap, so one path runs (the branch-free form ran both: +20 instructions
+    // per flush, and at nside >= 2048 some lane flushes at nearly every sample)
+    const unsigned pix = (unsigned)ckey_to_pix<NEST, OFF>(key, g);
     const unsigned sm = pix >> mg.sm_shift;
     const unsigned lp = pix & (unsigned)(mg.n_pix_submap - 1);
     const unsigned v = g2l[sm];
@@ -482,11 +495,12 @@ __device__ __forceinline__ void flush_lean(int key, double r0, double r1, double
     }
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool TMA, bool SCAN>
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool TMA, bool SCAN, bool QUEUE>
 __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
     pointing_to_map_kernel(const Chunk* __restrict__ chunks, int n_chunks, FusedArgs a, HealpixGeom g, KeyConsts kc,
                            unsigned long long* __restrict__ sched, const __grid_constant__ TmaMaps tm) {
     static_assert(!SCAN || !DEBUG, "the scan direction has no debug outputs");
+    static_assert(!QUEUE || (!SCAN && !DEBUG && !WIDE), "the flush queue: production map kernels, 32-bit keys");
     using P = typename PixT<WIDE>::T;
     constexpr bool OFF = kOff<NNZ, P>;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -634,15 +648,47 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
         load_slot<P>(sl, a, cur.d0 + lane, lane < cur.nrows, cur.d0);
         const double sgn_ds = (a.should_subtract ? -1.0 : 1.0) * a.data_scale;  // SCAN only
 
-        // A run ends: flush it (the lanes whose key changed; divergent).
-        auto flush_run = [&]() {
+        // A run ends: flush its scaled sums (the lanes whose key changed; divergent).
+        auto flush_run = [&](P key, double f0, double f1, double f2, int64_t det) {
             if (lean) {
-                flush_lean<NEST, NNZ, OFF>((int)sl.run_key, sl.r0 * sl.sI, sl.r1 * sl.sQ, sl.r2 * sl.sU, a, g, cm.g2l);
+                flush_lean<NEST, NNZ, OFF>((int)key, f0, f1, f2, a, g, cm.g2l);
             } else {
-                drain_general<NEST, NNZ, OFF, WIDE>(sl.run_key, sl.r0 * sl.sI, sl.r1 * sl.sQ, sl.r2 * sl.sU, a.zmap,
-                                                    a.map_f32, a.hit_submaps, mg.global2local, mg.sm_shift,
-                                                    mg.n_pix_submap, cm.g2l, cm.cached, a.gamma, a.hwp != nullptr,
-                                                    a.iau, sl.det, g);
+                drain_general<NEST, NNZ, OFF, WIDE>(key, f0, f1, f2, a.zmap, a.map_f32, a.hit_submaps,
+                                                    mg.global2local, mg.sm_shift, mg.n_pix_submap, cm.g2l, cm.cached,
+                                                    a.gamma, a.hwp != nullptr, a.iau, det, g);
+            }
+        };
+        // QUEUE: finished runs are pushed (one ballot, converged) into the warp's queue and
+        // flushed 32 at a time by all lanes, instead of by the few lanes whose key changed
+        // while the rest of the warp waits (better when runs are long enough
+        // that few lanes change key per sample, nside <= 2048)
+        int qn = 0;
+        const unsigned lt_mask = (1u << lane) - 1u;
+        auto drain = [&](int n) {
+            __syncwarp();
+            if (lane < n) {
+                const QEntry e = ws.q[lane];
+                flush_run((P)e.key, e.r0, e.r1, e.r2, (int64_t)cur.d0 + e.src);
+            }
+            __syncwarp();
+        };
+        auto push = [&](bool do_push, P key, double f0, double f1, double f2) {
+            const unsigned m = __ballot_sync(kFull, do_push);
+            if (m) {
+                const int np = __popc(m);
+                if (qn + np > kQ) {
+                    drain(qn);
+                    qn = 0;
+                }
+                if (do_push) {
+                    QEntry& e = ws.q[qn + __popc(m & lt_mask)];
+                    e.key = (int)key;
+                    e.src = lane;
+                    e.r0 = f0;
+                    e.r1 = f1;
+                    e.r2 = f2;
+                }
+                qn += np;
             }
         };
 
@@ -827,11 +873,21 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
                                 if (__ldg(&mg.global2local[smi]) < 0) atomicAdd(a.dropped, 1ull);
                             }
                         }
-                        // run-length aggregation: the run ends when the key changes
-                        if (key != sl.run_key) {
-                            if (sl.run_key >= 0) flush_run();
+                        // run-length aggregation: the run ends when the key changes (the sums are
+                        // reset once, before the flush, so the compiler keeps one copy of it)
+                        if constexpr (QUEUE) {
+                            const bool chg = key != sl.run_key;
+                            push(chg && sl.run_key >= 0, sl.run_key, sl.r0 * sl.sI, sl.r1 * sl.sQ, sl.r2 * sl.sU);
+                            if (chg) {
+                                sl.run_key = key;
+                                sl.r0 = sl.r1 = sl.r2 = 0.0;
+                            }
+                        } else if (key != sl.run_key) {
+                            const P old = sl.run_key;
+                            const double f0 = sl.r0 * sl.sI, f1 = sl.r1 * sl.sQ, f2 = sl.r2 * sl.sU;
                             sl.run_key = key;
                             sl.r0 = sl.r1 = sl.r2 = 0.0;
+                            if (old >= 0) flush_run(old, f0, f1, f2, sl.det);
                         }
                         sl.r0 += tod;
                         if (NNZ == 3) {
@@ -861,8 +917,12 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
             }
 
             if (nxt.item != cur.item) {
-                if constexpr (!SCAN) {
-                    if (sl.run_key >= 0) flush_run();  // the item's open runs
+                if constexpr (QUEUE) {
+                    push(sl.run_key >= 0, sl.run_key, sl.r0 * sl.sI, sl.r1 * sl.sQ, sl.r2 * sl.sU);  // open runs
+                    drain(qn);
+                    qn = 0;
+                } else if constexpr (!SCAN) {
+                    if (sl.run_key >= 0) flush_run(sl.run_key, sl.r0 * sl.sI, sl.r1 * sl.sQ, sl.r2 * sl.sU, sl.det);
                 }
                 if (nxt.item < 0) break;
                 load_slot<P>(sl, a, nxt.d0 + lane, lane < nxt.nrows, nxt.d0);
@@ -994,10 +1054,10 @@ void raise_smem_limit(K kern, bool* done_per_dev) {
     }
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool TMA, bool SCAN>
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool TMA, bool SCAN, bool QUEUE>
 cudaError_t launch_k(const WorkList& wl, const FusedArgs& a, const TmaMaps& tm, unsigned long long* sched,
                      cudaStream_t st) {
-    auto kern = pointing_to_map_kernel<NEST, NNZ, HWP, DEBUG, WIDE, TMA, SCAN>;
+    auto kern = pointing_to_map_kernel<NEST, NNZ, HWP, DEBUG, WIDE, TMA, SCAN, QUEUE>;
     static bool done[64] = {false};
     raise_smem_limit(kern, done);
     const size_t smem = fused_smem(a);
@@ -1022,23 +1082,33 @@ cudaError_t launch_k(const WorkList& wl, const FusedArgs& a, const TmaMaps& tm, 
     return cudaGetLastError();
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool SCAN>
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool SCAN, bool QUEUE = false>
 cudaError_t launch_t(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
     TmaMaps tm;
     if (make_tma_maps(a, &tm)) {
         t_fused_path = "tma";
-        return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, true, SCAN>(wl, a, tm, sched, st);
+        return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, true, SCAN, QUEUE>(wl, a, tm, sched, st);
     }
     std::memset(&tm, 0, sizeof(tm));
-    return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, false, SCAN>(wl, a, tm, sched, st);
+    return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, false, SCAN, QUEUE>(wl, a, tm, sched, st);
 }
 
 // nside <= 4096: 32-bit compact keys; beyond: 64-bit pixel keys
 constexpr int64_t kCompactMaxNside = 4096;
+// The converged flush queue (QUEUE kernels) for nside <= TB_QUEUE_MAX_NSIDE: measured slower than
+// the direct divergent flush on every benchmark config, so off by default.
+#ifndef TB_QUEUE_MAX_NSIDE
+#define TB_QUEUE_MAX_NSIDE 0  // measured r02v: C4 53.5 vs 52.3 ms, C3 0.477 vs 0.467 ms, C2 equal: off
+#endif
 
 template <bool NEST, int NNZ, bool HWP, bool DEBUG>
 cudaError_t dispatch_shape(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
     if (a.nside > kCompactMaxNside) return launch_t<NEST, NNZ, HWP, DEBUG, true, false>(wl, a, sched, st);
+#if TB_QUEUE_MAX_NSIDE > 0
+    if constexpr (!DEBUG) {
+        if (a.nside <= TB_QUEUE_MAX_NSIDE) return launch_t<NEST, NNZ, HWP, false, false, false, true>(wl, a, sched, st);
+    }
+#endif
     return launch_t<NEST, NNZ, HWP, DEBUG, false, false>(wl, a, sched, st);
 }
 
@@ -1164,7 +1234,7 @@ cudaError_t dispatch_scan(const WorkList& wl, const FusedArgs& a, unsigned long 
     if (wide) return hwp ? launch_t<NEST, NNZ, true, false, true, true>(wl, a, sched, st)
                          : launch_t<NEST, NNZ, false, false, true, true>(wl, a, sched, st);
     return hwp ? launch_t<NEST, NNZ, true, false, false, true>(wl, a, sched, st)
-               : launch_t<NEST, NNZ, false, false, false, true>(wl, a, sched, st);
+               : launch_t<NEST, NNZ, false, false, false, true>(wl, a, sched, st);  // (no queue: a scan gathers)
 }
 
 // Launch-side map geometry of the fused kernels: the submap count and whether the CTAs cache
