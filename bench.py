@@ -75,6 +75,9 @@ def parse():
     ap.add_argument("--shard", default="auto", choices=["auto", "det", "obs"],
                     help="N>1: detector blocks of one observation (strong scaling; auto for c4, c5m) or one "
                          "observation per rank (weak scaling; auto for the small configs)")
+    ap.add_argument("--graph", type=int, default=0,
+                    help="launch-bound configs (C1, SURVEY 8(d)): one step = a CUDA graph of G back-to-back "
+                         "(zero map + fused call)s, captured once and replayed")
     ap.add_argument("--reduce", default="auto", choices=["auto", "dense", "packed", "scatter"],
                     help="N>1 map reduction: dense all_reduce, all_reduce of the union of hit submaps (packed), "
                          "or the sparse distributed map domain (compact map + reduce_scatter, SURVEY 8(f) f3)")
@@ -358,6 +361,34 @@ def main():
             else:
                 _, reduced["bytes"] = tdist.reduce_map(zmap)
 
+    graph = None
+    if args.graph > 0:
+        if world > 1 or scan_map_in is not None:
+            raise SystemExit("--graph: single-GPU map workloads only")
+        step()  # the work list is cached before capture
+        torch.cuda.synchronize()
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph):
+            cs = torch.cuda.current_stream()
+            graws = [tuple(list(r[:-1]) + [cs.cuda_stream]) for r in raws]
+            for _ in range(args.graph):
+                zmap.zero_()
+                hits.zero_()
+                for raw in graws:
+                    if lib.toast_pointing_to_map(*raw) != 0:
+                        raise binding.ToastError(lib.toast_last_error().decode())
+        plain_step = step
+
+        def step(timed=False):  # noqa: F811  (one step = one replay of G calls)
+            if timed:
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+            graph.replay()
+            if timed:
+                b.record(stream)
+                kern_events.append((a, b))
+        del plain_step
+
     for _ in range(max(3, args.warmup)):
         step()
     torch.cuda.synchronize()
@@ -401,6 +432,10 @@ def main():
     ms = e0.elapsed_time(e1)
     kern_ms = statistics.mean(a.elapsed_time(b) for a, b in kern_events)  # per launch
     launches_per_step = len(obs) * (2 if scan_map_in is not None else 1)
+    if graph is not None:  # a replay holds G (zero + fused call)s: per call
+        kern_ms /= args.graph
+        det_samples *= args.graph
+        launches_per_step *= args.graph
     time.sleep(0.2)
     sampler.stop()
     clocks = sampler.summary(t_wall0, t_wall1)
@@ -417,10 +452,11 @@ def main():
     # ---- end to end through the public API, host (pinned) buffers, copies in the timed region
     e2e = None
     if not args.no_e2e:
-        e2e = run_e2e(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples, scan_map_in is not None)
+        e2e = run_e2e(args, obs, zmap, hits, g2l, world, stream, packed,
+                      total_det_samples / (args.graph if graph is not None else 1), scan_map_in is not None)
 
     # ---- roofline of the dominant kernel (the fused pointing->map kernel), per launch
-    det_per_launch = det_samples / len(obs)
+    det_per_launch = det_samples / len(obs) / (args.graph if graph is not None else 1)
     peak_meas, peak_src = fp64_peak()
     clk = clocks.get("sm_max_mhz") or 1965.0
     peak_nominal = SMS * DFMA_PER_SM_PER_CLK * 2 * clk * 1e6 / 1e12
@@ -483,6 +519,9 @@ def main():
                                    (" + map reduction" if world > 1 else ""),
                            "allreduce_bytes_per_step": reduced["bytes"], "allreduce_ms": ar_ms,
                            "staging": binding.last_fused_path(),
+                           "cuda_graph": (f"one step = one replay of a CUDA graph of {args.graph} x (zero map + "
+                                          "toast_pointing_to_map); roofline.kernel_ms per call includes the zeroing")
+                           if graph is not None else None,
                            "tod_source": "device counter hash (toast_synth_tod, bit-identical to synth.py)"
                            if name in DEVICE_TOD else "host synth.py"},
                 "clocks": clocks, "gpu_launches": args.steps * launches_per_step, "roofline": roofline}

@@ -148,8 +148,12 @@ int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, cudaStre
             (n == 0 || std::memcmp(c.intervals.data(), iv, sizeof(toast_interval_t) * n) == 0)) {
             c.last_use = ++g_cache_clock;
             if (c.uploaded && st != c.upload_stream) {
-                e = cudaStreamWaitEvent(st, c.uploaded, 0);
-                if (e != cudaSuccess) return cuda_fail(e, "cudaStreamWaitEvent on the work-list upload");
+                // (a capturing stream may not wait on uncaptured work: CUDA-graph capture of a call
+                // requires a prior call with the same intervals, synchronised — e.g. a warm-up)
+                cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+                e = cudaStreamIsCapturing(st, &cap);
+                if (e == cudaSuccess && cap == cudaStreamCaptureStatusNone) e = cudaStreamWaitEvent(st, c.uploaded, 0);
+                if (e != cudaSuccess) return cuda_fail(e, "ordering after the work-list upload");
             }
             out->wl = WorkList{c.d_chunks, c.n_chunks, c.n_samples};
             out->lock = std::move(lk);
@@ -665,8 +669,12 @@ int get_offset_views(const toast_interval_t* iv, int64_t n, int64_t step, cudaSt
             (n == 0 || std::memcmp(c.intervals.data(), iv, sizeof(toast_interval_t) * n) == 0)) {
             c.last_use = ++g_ocache_clock;
             if (c.uploaded && st != c.upload_stream) {
-                e = cudaStreamWaitEvent(st, c.uploaded, 0);
-                if (e != cudaSuccess) return cuda_fail(e, "cudaStreamWaitEvent on the offset-view upload");
+                // (a capturing stream may not wait on uncaptured work: CUDA-graph capture of a call
+                // requires a prior call with the same intervals, synchronised — e.g. a warm-up)
+                cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+                e = cudaStreamIsCapturing(st, &cap);
+                if (e == cudaSuccess && cap == cudaStreamCaptureStatusNone) e = cudaStreamWaitEvent(st, c.uploaded, 0);
+                if (e != cudaSuccess) return cuda_fail(e, "ordering after the offset-view upload");
             }
             *out = OffsetViews{c.d_arrays, c.d_arrays + n, (int)step};
             *lease = std::move(lk);

@@ -130,6 +130,12 @@ __device__ __forceinline__ void tma_2d_stream(void* dst, const CUtensorMap* m, i
 __device__ __forceinline__ void red_f64(double* p, double v) {
     asm volatile("red.global.add.f64 [%0], %1;" ::"l"(p), "d"(v) : "memory");
 }
+// predicated: no branch around the reduction (the flush stays straight-line code)
+__device__ __forceinline__ void red_f64_if(bool c, double* p, double v) {
+    asm volatile("{\n .reg .pred q;\n setp.ne.u32 q, %2, 0;\n @q red.global.add.f64 [%0], %1;\n}\n" ::"l"(p), "d"(v),
+                 "r"((unsigned)c)
+                 : "memory");
+}
 __device__ __forceinline__ void red_f32(float* p, float v) {
     asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
 }
@@ -485,6 +491,15 @@ __device__ __forceinline__ void flush_lean(int key, double r0, double r1, double
     const unsigned v = g2l[sm];
     g2l[sm] = (uint16_t)(v | kHitBit);  // idempotent: every writer stores the same value
     const unsigned loc = v & 0x7fffu;
+#ifdef TB_PRED_RED
+    const bool ok = loc != kNoLoc;
+    double* dst = a.zmap + (size_t)((loc << mg.sm_shift) + lp) * NNZ;
+    red_f64_if(ok, dst, r0);
+    if (NNZ == 3) {
+        red_f64_if(ok, dst + 1, r1);
+        red_f64_if(ok, dst + 2, r2);
+    }
+#else
     if (loc != kNoLoc) {
         double* dst = a.zmap + (size_t)((loc << mg.sm_shift) + lp) * NNZ;
         red_f64(dst, r0);
@@ -492,6 +507,29 @@ __device__ __forceinline__ void flush_lean(int key, double r0, double r1, double
             red_f64(dst + 1, r1);
             red_f64(dst + 2, r2);
         }
+    }
+#endif
+}
+
+// The lean flush as straight-line, PREDICATED code (no branch: executed by every lane at every
+// sample, the reductions and the hit-flag store predicated on `go`); a variant for scans where
+// some lane of the warp changes pixel at nearly every sample anyway (large nside).
+template <bool NEST, int NNZ, bool OFF>
+__device__ __forceinline__ void flush_lean_pred(bool go, int key, double r0, double r1, double r2,
+                                                const FusedArgs& a, const HealpixGeom& g, uint16_t* g2l) {
+    const MapGeom& mg = a.map;
+    const unsigned pix = (unsigned)ckey_to_pix_bf<NEST, OFF>(go ? key : 0, g);
+    const unsigned sm = pix >> mg.sm_shift;
+    const unsigned lp = pix & (unsigned)(mg.n_pix_submap - 1);
+    const unsigned v = g2l[sm];
+    if (go) g2l[sm] = (uint16_t)(v | kHitBit);
+    const unsigned loc = v & 0x7fffu;
+    const bool ok = go && loc != kNoLoc;
+    double* dst = a.zmap + (size_t)((loc << mg.sm_shift) + lp) * NNZ;
+    red_f64_if(ok, dst, r0);
+    if (NNZ == 3) {
+        red_f64_if(ok, dst + 1, r1);
+        red_f64_if(ok, dst + 2, r2);
     }
 }
 
@@ -882,6 +920,19 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
                                 sl.run_key = key;
                                 sl.r0 = sl.r1 = sl.r2 = 0.0;
                             }
+#ifdef TB_PRED_FLUSH
+                        } else if (lean) {
+                            // straight-line flush (see flush_lean_pred)
+                            const bool chg = key != sl.run_key;
+                            const double f0 = sl.r0 * sl.sI, f1 = sl.r1 * sl.sQ, f2 = sl.r2 * sl.sU;
+                            flush_lean_pred<NEST, NNZ, OFF>(chg && sl.run_key >= 0, (int)sl.run_key, f0, f1, f2, a, g,
+                                                            cm.g2l);
+                            const double keepr = chg ? 0.0 : 1.0;
+                            sl.r0 *= keepr;
+                            sl.r1 *= keepr;
+                            sl.r2 *= keepr;
+                            sl.run_key = key;
+#endif
                         } else if (key != sl.run_key) {
                             const P old = sl.run_key;
                             const double f0 = sl.r0 * sl.sI, f1 = sl.r1 * sl.sQ, f2 = sl.r2 * sl.sU;
