@@ -326,6 +326,8 @@ struct Slot {
     double px, py, ptt; // incremental longitude: projected direction and tt of the previous sample
     P run_key;          // key of the run being aggregated (-1: none)
     int64_t run_elem;   // SCAN: map element of the cached run (-1: none)
+    unsigned pend_addr; // SCAN: shared address of the sample whose TOD update is pending (~0: none)
+    double pend_c, pend_s;  // SCAN: its eta cal cos / r and 2 eta cal sin' / r
     int64_t det;
     bool ok;
 };
@@ -351,6 +353,8 @@ __device__ __forceinline__ void load_slot(Slot<P>& sl, const FusedArgs& a, int64
     sl.sU = 2.0 * usign * sl.sQ;
     sl.run_key = -1;
     sl.run_elem = -1;
+    sl.pend_addr = 0xffffffffu;
+    sl.pend_c = sl.pend_s = 0.0;
     sl.r0 = sl.r1 = sl.r2 = 0.0;
     sl.px = sl.py = sl.ptt = 0.0;  // dot = 0: the item's first sample takes the full arctangent
     sl.det = dd;
@@ -731,6 +735,26 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
         };
 
         int p = 0;
+        // SCAN: complete the pending sample's TOD update (t = data_scale sum_k m_k w_k)
+        auto scan_finish = [&]() {
+            if constexpr (SCAN) {
+                if (sl.pend_addr != 0xffffffffu) {
+                    double t = sl.r0 * a.cal;
+                    if (NNZ == 3) t = fma(sl.r1, sl.pend_c, fma(sl.r2, sl.pend_s, t));
+                    double v;
+                    if (a.should_zero) {
+                        v = sgn_ds * t;  // the old value is overwritten, never read (NaN-safe)
+                    } else {
+                        double old;
+                        asm volatile("ld.shared.f64 %0, [%1];" : "=d"(old) : "r"(sl.pend_addr));
+                        v = fma(sgn_ds, t, old);
+                    }
+                    asm volatile("st.shared.f64 [%0], %1;" ::"r"(sl.pend_addr), "d"(v) : "memory");
+                    sl.pend_addr = 0xffffffffu;
+                }
+            }
+        };
+
         while (true) {
             // successor block: next 16 samples of this item, or the first block of the next item
             const Blk nxt = successor(cur);
@@ -836,56 +860,49 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
                     P key = stage_b<NEST, NNZ, WIDE>(o, pixelise, g, kc);
                     if (!sl.ok) key = -1;
                     if constexpr (SCAN) {
-                        // gather the run's map values (cached per lane across the run), update the TOD
+                        // gather the run's map values (cached per lane across the run) and update the
+                        // TOD ONE SAMPLE LATER: the loads of a new run are in flight while the next
+                        // sample's pointing is computed (the update of sample k-1 runs here, before
+                        // sample k may start a new run)
+                        scan_finish();
                         if (key < 0) continue;
                         if (key != sl.run_key) {
                             sl.run_key = key;
                             sl.run_elem = locate(key_to_pixel<NEST, OFF, WIDE>(key, g), a, cm);
                             if (sl.run_elem >= 0) {
-                                double m0, m1 = 0.0, m2 = 0.0;
                                 if (a.map_f32) {
                                     const float* mp = reinterpret_cast<const float*>(a.mapdata) + sl.run_elem * NNZ;
-                                    m0 = __ldg(mp);
+                                    sl.r0 = __ldg(mp);
                                     if (NNZ == 3) {
-                                        m1 = __ldg(mp + 1);
-                                        m2 = __ldg(mp + 2);
+                                        sl.r1 = __ldg(mp + 1);
+                                        sl.r2 = __ldg(mp + 2);
                                     }
                                 } else {
                                     const double* mp = a.mapdata + sl.run_elem * NNZ;
-                                    m0 = __ldg(mp);
+                                    sl.r0 = __ldg(mp);
                                     if (NNZ == 3) {
-                                        m1 = __ldg(mp + 1);
-                                        m2 = __ldg(mp + 2);
+                                        sl.r1 = __ldg(mp + 1);
+                                        sl.r2 = __ldg(mp + 2);
                                     }
                                 }
-                                // fold the reading-R3 rotation / IAU sign into the gathered (m1, m2)
-                                if (NNZ == 3) {
-                                    if (a.iau) m2 = -m2;
+                                // reading R3 (a variant): t = m . (D R(-4 gamma) w) = (R(4 gamma) D m) . w;
+                                // gamma_rotate gives diag(1, -1) R(-4 gamma) (m1, -m2) = R(4 gamma) (m1, m2)
+                                if (NNZ == 3 && (a.iau || (a.gamma != nullptr && a.hwp != nullptr))) {
+                                    if (a.iau) sl.r2 = -sl.r2;
                                     if (a.gamma != nullptr && a.hwp != nullptr) {
-                                        // t = m . (D R(-4 gamma) w) = (R(4 gamma) D m) . w; gamma_rotate
-                                        // gives diag(1, -1) R(-4 gamma) (m1, -m2) = R(4 gamma) (m1, m2)
-                                        const double2 n = gamma_rotate(m1, -m2, a.gamma, 1, sl.det);
-                                        m1 = n.x;
-                                        m2 = n.y;
+                                        const double2 n = gamma_rotate(sl.r1, -sl.r2, a.gamma, 1, sl.det);
+                                        sl.r1 = n.x;
+                                        sl.r2 = n.y;
                                     }
                                 }
-                                sl.r0 = m0 * a.cal;
-                                sl.r1 = m1 * sl.etacal;
-                                sl.r2 = m2 * (2.0 * sl.etacal);
                             }
                         }
                         if (sl.run_elem < 0) continue;
-                        double t = sl.r0;
-                        if (NNZ == 3) t = fma(sl.r1 * o.invr, o.cw, fma(sl.r2 * o.invr, o.sw, t));
-                        double v;
-                        if (a.should_zero) {
-                            v = sgn_ds * t;  // the old value is overwritten, never read (NaN-safe)
-                        } else {
-                            double old;
-                            asm volatile("ld.shared.f64 %0, [%1];" : "=d"(old) : "r"(addr));
-                            v = fma(sgn_ds, t, old);
+                        sl.pend_addr = addr;
+                        if (NNZ == 3) {
+                            sl.pend_c = sl.etacal * (o.cw * o.invr);
+                            sl.pend_s = (2.0 * sl.etacal) * (o.sw * o.invr);
                         }
-                        asm volatile("st.shared.f64 [%0], %1;" ::"r"(addr), "d"(v) : "memory");
                     } else {
                         double tod;
                         asm volatile("ld.shared.f64 %0, [%1];" : "=d"(tod) : "r"(addr));
@@ -948,6 +965,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
                         }
                     }
                 }
+                scan_finish();  // the block's last pending update, before the write-back
                 __syncwarp();
                 if constexpr (SCAN) {
                     // write back the processed columns of the tile (two rows per warp instruction,
