@@ -106,6 +106,11 @@ class ClockSampler:
                                          stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
         except (FileNotFoundError, OSError):
             self.proc = None
+            return
+        # nvidia-smi can take a second to print its first sample: the timed region starts after it
+        t0 = time.time()
+        while time.time() - t0 < 5.0 and os.path.getsize(self.path) == 0:
+            time.sleep(0.05)
 
     def stop(self):
         if self.proc is not None:
@@ -330,7 +335,23 @@ def main():
     raws = [o.dw.raw_args(stream, zmap=zmap) for o in obs]
     raws = [tuple(list(r[:19]) + [hits.data_ptr()] + list(r[20:])) for r in raws]
 
-    packed = world > 1 and (args.reduce == "packed" or (args.reduce == "auto" and zmap.numel() * 8 > (256 << 20)))
+    # f3 sparse map domain (--reduce scatter): one pointing pass marks the hit submaps (TOAST computes
+    # its pixel distribution once per data set), the map then holds storage for the union of hit
+    # submaps only; N > 1 reduce-scatters it (each rank keeps its owned block)
+    own = None
+    if args.reduce == "scatter":
+        for raw in raws:
+            if lib.toast_pointing_to_map(*raw) != 0:
+                raise binding.ToastError(lib.toast_last_error().decode())
+        hits_all = tdist.union_hit_submaps(hits) if world > 1 else hits
+        g2l, n_hit = tdist.compact_global2local(hits_all)
+        own = tdist.MapOwnership.make(n_hit, world)
+        zmap = tdist.alloc_compact_map(own, nps, nnz, dev)
+        raws = [o.dw.raw_args(stream, zmap=zmap, global2local=g2l) for o in obs]
+        raws = [tuple(list(r[:19]) + [hits.data_ptr()] + list(r[20:])) for r in raws]
+        torch.cuda.synchronize()
+
+    packed = own is None and world > 1 and (args.reduce == "packed" or (args.reduce == "auto" and zmap.numel() * 8 > (256 << 20)))
     reduced = {"bytes": 0}
     kern_events = []  # (start, end) of every fused map launch in the timed region
 
@@ -355,7 +376,9 @@ def main():
                 b.record(stream)
                 kern_events.append((a, b))
         if world > 1:
-            if packed:
+            if own is not None:
+                _, reduced["bytes"] = tdist.reduce_scatter_map(zmap, own)
+            elif packed:
                 tdist.union_hit_submaps(hits)
                 _, reduced["bytes"] = tdist.reduce_map(zmap, hit_submaps=hits, global2local=g2l)
             else:
@@ -404,7 +427,9 @@ def main():
         dist.barrier()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
-        if packed:
+        if own is not None:
+            tdist.reduce_scatter_map(zmap, own)
+        elif packed:
             tdist.union_hit_submaps(hits)
             tdist.reduce_map(zmap, hit_submaps=hits, global2local=g2l)
         else:
@@ -453,7 +478,7 @@ def main():
     e2e = None
     if not args.no_e2e:
         e2e = run_e2e(args, obs, zmap, hits, g2l, world, stream, packed,
-                      total_det_samples / (args.graph if graph is not None else 1), scan_map_in is not None)
+                      total_det_samples / (args.graph if graph is not None else 1), scan_map_in is not None, own)
 
     # ---- roofline of the dominant kernel (the fused pointing->map kernel), per launch
     det_per_launch = det_samples / len(obs) / (args.graph if graph is not None else 1)
@@ -517,6 +542,9 @@ def main():
                            "step": "zero map + " + ("(pointing_to_tod + pointing_to_map) per observation"
                                                     if scan_map_in is not None else "toast_pointing_to_map") +
                                    (" + map reduction" if world > 1 else ""),
+                           "map_domain": (f"compact: {own.n_hit} hit submaps of {n_submap} (dist.compact_global2local)"
+                                          + (", NCCL reduce_scatter" if world > 1 else "")) if own is not None
+                           else "dense",
                            "allreduce_bytes_per_step": reduced["bytes"], "allreduce_ms": ar_ms,
                            "staging": binding.last_fused_path(),
                            "cuda_graph": (f"one step = one replay of a CUDA graph of {args.graph} x (zero map + "
@@ -534,7 +562,7 @@ def main():
         dist.destroy_process_group()
 
 
-def run_e2e(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples, with_scan):
+def run_e2e(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples, with_scan, own=None):
     """Same metric through the public API with host buffers: every step copies the step's inputs
     from pinned host memory (the TOD in 256-detector blocks through two device staging buffers,
     overlapped with the fused kernel: streaming.Streamer) and reads the map back."""
@@ -575,7 +603,9 @@ def run_e2e(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples
                                det_flag_mask=o.w.det_flag_mask, shared_flag_mask=o.w.shared_flag_mask,
                                hit_submaps=hits, stream=stream)
         if world > 1:
-            if packed:
+            if own is not None:
+                tdist.reduce_scatter_map(zmap, own)
+            elif packed:
                 tdist.union_hit_submaps(hits)
                 tdist.reduce_map(zmap, hit_submaps=hits, global2local=g2l)
             else:

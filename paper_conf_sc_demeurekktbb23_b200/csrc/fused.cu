@@ -50,6 +50,10 @@ namespace {
 #ifndef TB_FUSED_MINB
 #define TB_FUSED_MINB 2  // resident CTAs per SM the register allocation is bounded for
 #endif
+#ifndef TB_ORDER_W
+#define TB_ORDER_W 0
+#endif
+constexpr int kOrderW = TB_ORDER_W;
 constexpr int kWarps = 8;  // warps per CTA
 constexpr int kBlk = 16;   // samples per block
 constexpr unsigned kFull = 0xffffffffu;
@@ -589,12 +593,27 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
     // Lane 0 fetches the NEXT item id and its chunk descriptor one item ahead (issued at an item
     // switch, consumed at the next one), so neither latency is on the critical path.
     int pend_item = -1, pend_first = 0, pend_count = 0;
+    // item -> (chunk, detector group): windows of kOrderW chunks, group-major inside a window
+    // (kOrderW = 0: chunk-major, all groups of a chunk in a row)
+    auto item_chunk = [&](int item, int& grp) -> int {
+        if (kOrderW <= 0) {
+            const int c = item / n_groups;
+            grp = item - c * n_groups;
+            return c;
+        }
+        const int win = item / (kOrderW * n_groups);
+        const int r = item - win * kOrderW * n_groups;
+        const int wc = min(kOrderW, n_chunks - win * kOrderW);
+        grp = r / wc;
+        return win * kOrderW + (r - grp * wc);
+    };
     auto prefetch_item = [&]() {
         if (lane == 0) {
             const unsigned long long it = atomicAdd(sched, 1ull);
             pend_item = it < (unsigned long long)n_items ? (int)it : -1;
             if (pend_item >= 0) {
-                const Chunk ch = chunks[pend_item / n_groups];
+                int grp;
+                const Chunk ch = chunks[item_chunk(pend_item, grp)];
                 pend_first = (int)ch.first;
                 pend_count = ch.count;
             }
@@ -609,8 +628,9 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
             bk.d0 = bk.s0 = bk.s_end = bk.nb = bk.nrows = bk.k0 = 0;
             return bk;
         }
-        const int c = bk.item / n_groups;
-        bk.d0 = (bk.item - c * n_groups) * 32;
+        int grp;
+        (void)item_chunk(bk.item, grp);
+        bk.d0 = grp * 32;
         bk.nrows = min(32, (int)a.n_det - bk.d0);
         // boxes start at multiples of 16 samples (a TMA box must start 16-byte aligned in every
         // staged row; the u8 flag rows need that); a chunk's first block processes k0 .. 15 only

@@ -72,7 +72,7 @@ class DeviceWorkload:
             shared_flag_mask=w.shared_flag_mask, hit_submaps=self.hit_submaps if hit_submaps is None else hit_submaps,
             pixels_out=pixels_out, weights_out=weights_out, stream=stream, gamma=gamma, iau=iau, dropped=dropped)
 
-    def raw_args(self, stream=None, zmap=None, det_data=None):
+    def raw_args(self, stream=None, zmap=None, det_data=None, global2local=None):
         """Pre-marshalled argument tuple of toast_pointing_to_map (no per-call Python checks)."""
         w = self.w
         st = (stream or torch.cuda.current_stream()).cuda_stream
@@ -81,5 +81,5 @@ class DeviceWorkload:
         return (p(self.fp_quats), p(self.boresight), p(self.hwp), p(self.epsilon), float(w.cal), p(self.det_scale),
                 p(self.det_data if det_data is None else det_data), p(self.det_flags), w.det_flag_mask,
                 p(self.shared_flags), w.shared_flag_mask, iv.ctypes.data if len(iv) else None, len(iv), w.nside,
-                int(w.nest), w.nnz, p(self.global2local), w.n_pix_submap, p(self.zmap if zmap is None else zmap),
+                int(w.nest), w.nnz, p(self.global2local if global2local is None else global2local), w.n_pix_submap, p(self.zmap if zmap is None else zmap),
                 p(self.hit_submaps), None, None, w.n_det, w.n_samp, st)
