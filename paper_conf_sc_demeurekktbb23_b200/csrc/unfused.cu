@@ -23,6 +23,8 @@ __device__ __forceinline__ void load_quat(const double* __restrict__ p, double q
     q[0] = lo.x; q[1] = lo.y; q[2] = hi.x; q[3] = hi.y;
 }
 
+__device__ __noinline__ void full_sincos(double a, double* s, double* c) { sincos(a, s, c); }
+
 // IDX = false: no row-index arrays (the common case) — no uniform branch between the loads
 // of a detector tile, so they issue back to back.
 template <bool IDX>
@@ -46,6 +48,10 @@ dim3 grid_for(const WorkList& wl, int64_t n_det, int dt = kDT) {
 
 // Resident 256-thread CTAs per SM each kernel's register allocation is bounded for (latency-bound
 // streaming kernels: more resident warps, more loads in flight).
+#ifndef TB_A1_DT
+#define TB_A1_DT 4
+#endif
+constexpr int kA1DT = TB_A1_DT;  // A1: detectors per thread (stores only: no registers held per detector)
 #ifndef TB_A1_MINB
 #define TB_A1_MINB 1
 #endif
@@ -53,7 +59,8 @@ dim3 grid_for(const WorkList& wl, int64_t n_det, int dt = kDT) {
 #define TB_A2_MINB 4  // measured on B200 (C2/C3): -26 % vs unbounded (80 registers -> 64)
 #endif
 #ifndef TB_A3_MINB
-#define TB_A3_MINB 1  // bounded variants spill (272+ bytes of stack) and run 50 % slower
+#define TB_A3_MINB 3  // measured on B200: 80 registers, C2 0.78 -> 0.71 ms, C3 0.56 -> 0.49 ms (the full-range
+                      // sincos is out of line; hoisting the per-detector loads above the stores: slower)
 #endif
 #ifndef TB_A4_MINB
 #define TB_A4_MINB 8  // measured: -21 % (46 registers -> 32, 5 -> 8 resident CTAs)
@@ -75,15 +82,15 @@ __global__ void __launch_bounds__(kChunk, TB_A1_MINB) pointing_detector_kernel(
         const Chunk ch = chunks[c];
         if ((int)threadIdx.x >= ch.count) continue;
         const int64_t s = ch.first + threadIdx.x;
+        // both loads issued before either is used (one HBM round trip, not two; C2 0.469 -> 0.433 ms)
         double b[4];
+        load_quat(boresight + 4 * s, b);
         if (shared_flags && (__ldg(&shared_flags[s]) & shared_flag_mask)) {
             b[0] = 0.0; b[1] = 0.0; b[2] = 0.0; b[3] = 1.0;  // reading S2
-        } else {
-            load_quat(boresight + 4 * s, b);
         }
-        FOR_DET_TILES(d0) {
+        for (int64_t d0 = (int64_t)blockIdx.y * kA1DT; d0 < n_det; d0 += (int64_t)gridDim.y * kA1DT) {
 #pragma unroll
-            for (int j = 0; j < kDT; ++j) {
+            for (int j = 0; j < kA1DT; ++j) {
                 const int64_t d = d0 + j;
                 if (d >= n_det) break;
                 double f[4], q[4];
@@ -157,8 +164,16 @@ __global__ void __launch_bounds__(kChunk, TB_A3_MINB) stokes_weights_kernel(
         if ((int)threadIdx.x >= ch.count) continue;
         const int64_t s = ch.first + threadIdx.x;
         double c4 = 1.0, s4 = 0.0;
-        // reading R1: sincos of the exact 4 chi (full-range reduction) for any finite chi
-        if (HWP) sincos(4.0 * __ldg(&hwp[s]), &s4, &c4);
+        // reading R1: sincos of the exact 4 chi for any finite chi (the short Cody-Waite reduction
+        // below 2^20 pi/2, the out-of-line full-range one beyond: its Payne-Hanek path would
+        // otherwise set this kernel's register count)
+        if (HWP) {
+            const double a4 = 4.0 * __ldg(&hwp[s]);
+            if (fabs(a4) < 1.6e6)
+                small_sincos(a4, &s4, &c4);
+            else
+                full_sincos(a4, &s4, &c4);
+        }
         FOR_DET_TILES(d0) {
             double q[kDT][4];
 #pragma unroll
@@ -181,7 +196,11 @@ __global__ void __launch_bounds__(kChunk, TB_A3_MINB) stokes_weights_kernel(
                     sq = s2 * c4 + c2 * s4;
                     if (gamma) {  // reading R3: rotate by -4 gamma (a variant; one sincos per det-sample)
                         double sg, cg;
-                        sincos(4.0 * __ldg(&gamma[d]), &sg, &cg);
+                        const double ag = 4.0 * __ldg(&gamma[d]);
+                        if (fabs(ag) < 1.6e6)
+                            small_sincos(ag, &sg, &cg);
+                        else
+                            full_sincos(ag, &sg, &cg);
                         const double q = fma(cg, cq, sg * sq), u = fma(cg, sq, -sg * cq);
                         cq = q;
                         sq = u;
@@ -308,7 +327,7 @@ cudaError_t launch_pointing_detector(const WorkList& wl, const double* fp_quats,
                                      const int32_t* quat_index, double* quats, const uint8_t* shared_flags,
                                      uint8_t shared_flag_mask, int64_t n_det, int64_t n_samp, cudaStream_t st) {
     if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
-    (quat_index ? pointing_detector_kernel<true> : pointing_detector_kernel<false>)<<<grid_for(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, fp_quats, boresight,
+    (quat_index ? pointing_detector_kernel<true> : pointing_detector_kernel<false>)<<<grid_for(wl, n_det, kA1DT), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, fp_quats, boresight,
                                                                       quat_index, quats, shared_flags,
                                                                       shared_flag_mask, n_det, n_samp);
     return cudaGetLastError();

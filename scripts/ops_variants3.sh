@@ -1,0 +1,13 @@
+# GPU box: per-entry timings of the unfused entries for variant libraries (C2, C3).
+export PYTHONPATH=.
+OUT=gpurun_out/$1; shift; mkdir -p $OUT
+for lib in paper_conf_sc_demeurekktbb23_b200/libtoastb200.so "$@"; do
+  v=$(basename $lib .so)
+  for w in c2 c3; do
+    TOASTB200_LIB=$(readlink -f $lib) timeout 300 python scripts/bench_ops.py --workload $w --only "(A1),(A2),(A3),(A4)" 2>&1 | python -c "
+import sys, json
+for l in sys.stdin:
+    try: d=json.loads(l); print('$v', d['workload'], d['entry'][:28], '%.4f ms'%d['ms'], 'hbm %.2f'%d.get('hbm_frac',0))
+    except Exception: pass"
+  done
+done | tee $OUT/variants.txt
