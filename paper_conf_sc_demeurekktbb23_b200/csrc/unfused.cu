@@ -108,7 +108,8 @@ __global__ void __launch_bounds__(kChunk, TB_A1_MINB) pointing_detector_kernel(
 
 // ----------------------------------------------------------------------------- A2
 
-template <bool NEST, bool IDX>
+// SMALL: nside <= 8192, the 32-bit integer pixel arithmetic (loc2pix32)
+template <bool NEST, bool IDX, bool SMALL>
 __global__ void __launch_bounds__(kChunk, TB_A2_MINB) pixels_healpix_kernel(
     const Chunk* __restrict__ chunks, int64_t n_chunks, const int32_t* __restrict__ quat_index,
     const double* __restrict__ quats, const uint8_t* __restrict__ shared_flags, uint8_t shared_flag_mask,
@@ -137,7 +138,7 @@ __global__ void __launch_bounds__(kChunk, TB_A2_MINB) pixels_healpix_kernel(
                     const double dx = 2.0 * (q[j][0] * q[j][2] + q[j][1] * q[j][3]);
                     const double dy = 2.0 * (q[j][1] * q[j][2] - q[j][0] * q[j][3]);
                     const double dz = 1.0 - 2.0 * (q[j][0] * q[j][0] + q[j][1] * q[j][1]);
-                    pix = vec2pix<NEST>(g, dx, dy, dz);
+                    pix = SMALL ? (int64_t)loc2pix32<NEST>(g, dz, phi_to_tt(dx, dy), dx, dy) : vec2pix<NEST>(g, dx, dy, dz);
                 }
                 if (in) __stcs(&pixels[row_of<IDX>(pixel_index, d) * n_samp + s], (long long)pix);
                 if (hit_submaps) {
@@ -339,14 +340,13 @@ cudaError_t launch_pixels_healpix(const WorkList& wl, const int32_t* quat_index,
                                   int nest, int64_t n_det, int64_t n_samp, cudaStream_t st) {
     if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
     const HealpixGeom g = make_geom(nside);
-    if (nest)
-        (quat_index || pixel_index ? pixels_healpix_kernel<true, true> : pixels_healpix_kernel<true, false>)<<<grid_for(wl, n_det), kChunk, 0, st>>>(
-            wl.chunks, wl.n_chunks, quat_index, quats, shared_flags, shared_flag_mask, pixel_index, pixels,
-            hit_submaps, n_pix_submap, g, n_det, n_samp);
-    else
-        (quat_index || pixel_index ? pixels_healpix_kernel<false, true> : pixels_healpix_kernel<false, false>)<<<grid_for(wl, n_det), kChunk, 0, st>>>(
-            wl.chunks, wl.n_chunks, quat_index, quats, shared_flags, shared_flag_mask, pixel_index, pixels,
-            hit_submaps, n_pix_submap, g, n_det, n_samp);
+    const bool idx = quat_index || pixel_index, small = nside <= 8192;
+    auto k = nest ? (idx ? (small ? pixels_healpix_kernel<true, true, true> : pixels_healpix_kernel<true, true, false>)
+                         : (small ? pixels_healpix_kernel<true, false, true> : pixels_healpix_kernel<true, false, false>))
+                  : (idx ? (small ? pixels_healpix_kernel<false, true, true> : pixels_healpix_kernel<false, true, false>)
+                         : (small ? pixels_healpix_kernel<false, false, true> : pixels_healpix_kernel<false, false, false>));
+    k<<<grid_for(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, quat_index, quats, shared_flags, shared_flag_mask,
+                                              pixel_index, pixels, hit_submaps, n_pix_submap, g, n_det, n_samp);
     return cudaGetLastError();
 }
 
