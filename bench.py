@@ -478,7 +478,7 @@ def main():
     e2e = None
     if not args.no_e2e:
         e2e = run_e2e(args, obs, zmap, hits, g2l, world, stream, packed,
-                      total_det_samples / (args.graph if graph is not None else 1), scan_map_in is not None, own)
+                      total_det_samples / (args.graph if graph is not None else 1), scan_map_in, own)
 
     # ---- roofline of the dominant kernel (the fused pointing->map kernel), per launch
     det_per_launch = det_samples / len(obs) / (args.graph if graph is not None else 1)
@@ -570,9 +570,8 @@ def run_e2e(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples
     import torch.distributed as dist
     from paper_conf_sc_demeurekktbb23_b200 import dist as tdist
     from paper_conf_sc_demeurekktbb23_b200.streaming import HostInputs, Streamer
-    if with_scan:
-        return {"value": None, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0,
-                "note": "round-trip workloads scan into the device TOD; e2e is measured on c1-c5"}
+    if with_scan is not None:
+        return run_e2e_round_trip(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples, own, with_scan)
     hosts, streamers = [], []
     try:
         for o in obs:
@@ -630,6 +629,83 @@ def run_e2e(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples
             "d2h_bytes_per_step": d2h, "steps": steps,
             "path": "streaming.Streamer -> binding.pointing_to_map (ctypes -> toast_pointing_to_map), TOD in "
                     "256-detector blocks from pinned host memory, copy of block b+1 overlapping the kernel on b"}
+
+
+def run_e2e_round_trip(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples, own, scan_map_in):
+    """e2e of the round-trip workloads (c3rt, c5m): every step copies the input map and each
+    observation's pointing inputs (focal plane, boresight, HWP, flags; the TOD is the scan's
+    output and never leaves the device) from pinned host memory, scans and accumulates through
+    the public API, and reads the map back."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_demeurekktbb23_b200 import binding
+    from paper_conf_sc_demeurekktbb23_b200 import dist as tdist
+
+    def pin(t):
+        if t is None:
+            return None
+        h = torch.empty(t.shape, dtype=t.dtype, pin_memory=True)
+        h.copy_(t)
+        return h
+    try:
+        names = ("fp_quats", "boresight", "epsilon", "det_scale", "hwp", "det_flags", "shared_flags")
+        hosts = [{k: pin(getattr(o.dw, k)) for k in names} for o in obs]
+        host_in = pin(scan_map_in)
+        host_map = torch.empty(zmap.shape, dtype=torch.float64).pin_memory()
+    except RuntimeError as e:  # pinned host memory exhausted
+        return {"value": None, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0,
+                "note": f"pinned host buffers unavailable: {str(e)[:120]}"}
+    dev_in = torch.empty_like(scan_map_in)
+    h2d = host_in.numel() * 8 + sum(t.numel() * t.element_size() for h in hosts for t in h.values() if t is not None)
+    d2h = host_map.numel() * 8
+
+    def e2e_step():
+        dev_in.copy_(host_in, non_blocking=True)
+        zmap.zero_()
+        hits.zero_()
+        for o, h in zip(obs, hosts):
+            for k, t in h.items():
+                if t is not None:
+                    getattr(o.dw, k).copy_(t, non_blocking=True)
+            w, dw = o.w, o.dw
+            binding.pointing_to_tod(dw.fp_quats, dw.boresight, dw.epsilon, w.cal, dw.intervals, w.nside, w.nest, w.nnz,
+                                    g2l, w.n_pix_submap, dev_in, dw.det_data, should_zero=True, hwp=dw.hwp,
+                                    shared_flags=dw.shared_flags, shared_flag_mask=w.shared_flag_mask, stream=stream)
+            binding.pointing_to_map(dw.fp_quats, dw.boresight, dw.epsilon, w.cal, dw.det_scale, dw.det_data,
+                                    dw.intervals, w.nside, w.nest, w.nnz, g2l, w.n_pix_submap, zmap, hwp=dw.hwp,
+                                    det_flags=dw.det_flags, det_flag_mask=w.det_flag_mask,
+                                    shared_flags=dw.shared_flags, shared_flag_mask=w.shared_flag_mask,
+                                    hit_submaps=hits, stream=stream)
+        if world > 1:
+            if own is not None:
+                tdist.reduce_scatter_map(zmap, own)
+            elif packed:
+                tdist.union_hit_submaps(hits)
+                tdist.reduce_map(zmap, hit_submaps=hits, global2local=g2l)
+            else:
+                tdist.reduce_map(zmap)
+        host_map.copy_(zmap, non_blocking=True)
+
+    e2e_step()
+    torch.cuda.synchronize()
+    steps = max(2, min(args.steps, 5))
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    if world > 1:
+        dist.barrier()
+    a.record(stream)
+    for _ in range(steps):
+        e2e_step()
+    b.record(stream)
+    torch.cuda.synchronize()
+    ms = torch.tensor([a.elapsed_time(b)], dtype=torch.float64, device=zmap.device)
+    if world > 1:
+        dist.all_reduce(ms, op=dist.ReduceOp.MAX)
+    ms = float(ms[0])
+    return {"value": total_det_samples * steps / (ms / 1e3), "unit": UNIT, "h2d_bytes_per_step": h2d,
+            "d2h_bytes_per_step": d2h, "steps": steps,
+            "path": "binding.pointing_to_tod -> binding.pointing_to_map per observation (ctypes -> C-ABI), the input "
+                    "map and every observation's pointing inputs copied from pinned host memory each step, the "
+                    "map read back"}
 
 
 if __name__ == "__main__":
