@@ -267,6 +267,65 @@ __device__ __forceinline__ void add_run(int64_t elem, double r0, double r1, doub
 
 // The general run flush (64-bit keys, non-power-of-two submaps, uncached global2local, fp32
 // maps, the reading-R3 rotation), out of line so that the hot loop's code stays small.
+// SCAN, general case (non-power-of-two submap, uncached global2local, fp32 map, gamma / IAU):
+// the map element of `key` and its values, folded for reading R3.  Out of line, so the hot
+// loop keeps only the lean gather.
+struct Gathered {
+    double m0, m1, m2;
+    int64_t elem;
+};
+template <bool NEST, int NNZ, bool OFF, bool WIDE>
+__device__ __noinline__ Gathered gather_general(typename PixT<WIDE>::T key, const double* mapdata, int map_f32,
+                                                const int64_t* global2local, int sm_shift, int64_t n_pix_submap,
+                                                uint16_t* g2l, bool cached, const double* gamma, bool have_hwp,
+                                                int iau, int64_t det, HealpixGeom g) {
+    Gathered r{0.0, 0.0, 0.0, -1};
+    const int64_t pix = key_to_pixel<NEST, OFF, WIDE>(key, g);
+    int64_t sm, lp;
+    if (sm_shift >= 0) {
+        sm = pix >> sm_shift;
+        lp = pix & (n_pix_submap - 1);
+    } else {
+        sm = pix / n_pix_submap;
+        lp = pix - sm * n_pix_submap;
+    }
+    int64_t loc;
+    if (cached) {
+        const unsigned l = g2l[sm] & 0x7fffu;
+        loc = l == kNoLoc ? -1 : (int64_t)l;
+    } else {
+        loc = __ldg(&global2local[sm]);
+    }
+    if (loc < 0) return r;
+    r.elem = loc * n_pix_submap + lp;
+    if (map_f32) {
+        const float* mp = reinterpret_cast<const float*>(mapdata) + r.elem * NNZ;
+        r.m0 = __ldg(mp);
+        if (NNZ == 3) {
+            r.m1 = __ldg(mp + 1);
+            r.m2 = __ldg(mp + 2);
+        }
+    } else {
+        const double* mp = mapdata + r.elem * NNZ;
+        r.m0 = __ldg(mp);
+        if (NNZ == 3) {
+            r.m1 = __ldg(mp + 1);
+            r.m2 = __ldg(mp + 2);
+        }
+    }
+    // reading R3 (a variant): t = m . (D R(-4 gamma) w) = (R(4 gamma) D m) . w;
+    // gamma_rotate gives diag(1, -1) R(-4 gamma) (m1, -m2) = R(4 gamma) (m1, m2)
+    if (NNZ == 3) {
+        if (iau) r.m2 = -r.m2;
+        if (gamma != nullptr && have_hwp) {
+            const double2 n = gamma_rotate(r.m1, -r.m2, gamma, 1, det);
+            r.m1 = n.x;
+            r.m2 = n.y;
+        }
+    }
+    return r;
+}
+
 template <bool NEST, int NNZ, bool OFF, bool WIDE>
 __device__ __noinline__ void drain_general(typename PixT<WIDE>::T key, double r0, double r1, double r2, double* zmap,
                                            int map_f32, uint8_t* hit_submaps, const int64_t* global2local,
@@ -573,6 +632,8 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
     const CtaMem cm{s_g2l, mg.cache_g2l && !s_nocache};
     const bool lean = !WIDE && mg.sm_shift >= 0 && cm.cached && !a.map_f32 &&
                       !(a.gamma != nullptr && a.hwp != nullptr) && a.hit_submaps != nullptr;
+    const bool scan_lean = SCAN && !WIDE && mg.sm_shift >= 0 && cm.cached && !a.map_f32 && !a.iau &&
+                           !(a.gamma != nullptr && a.hwp != nullptr);
 
     const int n_groups = (int)((a.n_det + 31) / 32);
     const int n_items = n_chunks * n_groups;
@@ -888,33 +949,28 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
                         if (key < 0) continue;
                         if (key != sl.run_key) {
                             sl.run_key = key;
-                            sl.run_elem = locate(key_to_pixel<NEST, OFF, WIDE>(key, g), a, cm);
-                            if (sl.run_elem >= 0) {
-                                if (a.map_f32) {
-                                    const float* mp = reinterpret_cast<const float*>(a.mapdata) + sl.run_elem * NNZ;
-                                    sl.r0 = __ldg(mp);
-                                    if (NNZ == 3) {
-                                        sl.r1 = __ldg(mp + 1);
-                                        sl.r2 = __ldg(mp + 2);
-                                    }
-                                } else {
-                                    const double* mp = a.mapdata + sl.run_elem * NNZ;
+                            if (scan_lean) {
+                                // 32-bit decode, cached global2local, one 3-load gather
+                                const unsigned pix = (unsigned)ckey_to_pix<NEST, OFF>((int)key, g);
+                                const unsigned loc = cm.g2l[pix >> mg.sm_shift] & 0x7fffu;
+                                const unsigned elem = (loc << mg.sm_shift) + (pix & (unsigned)(mg.n_pix_submap - 1));
+                                sl.run_elem = loc == kNoLoc ? -1 : (int64_t)elem;
+                                if (loc != kNoLoc) {
+                                    const double* mp = a.mapdata + (size_t)elem * NNZ;
                                     sl.r0 = __ldg(mp);
                                     if (NNZ == 3) {
                                         sl.r1 = __ldg(mp + 1);
                                         sl.r2 = __ldg(mp + 2);
                                     }
                                 }
-                                // reading R3 (a variant): t = m . (D R(-4 gamma) w) = (R(4 gamma) D m) . w;
-                                // gamma_rotate gives diag(1, -1) R(-4 gamma) (m1, -m2) = R(4 gamma) (m1, m2)
-                                if (NNZ == 3 && (a.iau || (a.gamma != nullptr && a.hwp != nullptr))) {
-                                    if (a.iau) sl.r2 = -sl.r2;
-                                    if (a.gamma != nullptr && a.hwp != nullptr) {
-                                        const double2 n = gamma_rotate(sl.r1, -sl.r2, a.gamma, 1, sl.det);
-                                        sl.r1 = n.x;
-                                        sl.r2 = n.y;
-                                    }
-                                }
+                            } else {
+                                const Gathered gm = gather_general<NEST, NNZ, OFF, WIDE>(
+                                    key, a.mapdata, a.map_f32, mg.global2local, mg.sm_shift, mg.n_pix_submap, cm.g2l,
+                                    cm.cached, a.gamma, a.hwp != nullptr, a.iau, sl.det, g);
+                                sl.run_elem = gm.elem;
+                                sl.r0 = gm.m0;
+                                sl.r1 = gm.m1;
+                                sl.r2 = gm.m2;
                             }
                         }
                         if (sl.run_elem < 0) continue;
