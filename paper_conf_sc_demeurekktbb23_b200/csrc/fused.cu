@@ -42,10 +42,13 @@
 
 #include "device_math.cuh"
 #include "internal.h"
+#include "tma.cuh"
 
 namespace toastb200 {
 
 namespace {
+
+using namespace tma;
 
 #ifndef TB_FUSED_MINB
 #define TB_FUSED_MINB 2  // resident CTAs per SM the register allocation is bounded for
@@ -58,29 +61,6 @@ constexpr int kWarps = 8;  // warps per CTA
 constexpr int kBlk = 16;   // samples per block
 constexpr unsigned kFull = 0xffffffffu;
 
-__device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
-
-__device__ __forceinline__ void cp_async8(unsigned dst, const void* gmem) {
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(dst), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async8_pol(unsigned dst, const void* gmem, uint64_t pol) {
-    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 8, %2;\n" ::"r"(dst), "l"(gmem), "l"(pol)
-                 : "memory");
-}
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
-
-// L2 evict-first policy for the streamed-once inputs (TOD, det flags): they must not push the
-// map lines being accumulated out of L2.
-__device__ __forceinline__ uint64_t evict_first_policy() {
-    uint64_t pol;
-    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;\n" : "=l"(pol));
-    return pol;
-}
-
 // ----------------------------------------------------------------------------- TMA
 struct alignas(64) TmaMaps {
     CUtensorMap tod;   // f64 [n_det][n_samp], box {16, 32}, SWIZZLE_128B
@@ -89,60 +69,6 @@ struct alignas(64) TmaMaps {
     CUtensorMap hwp;   // f64 [n_samp],        box {16}
     CUtensorMap sflg;  // u8  [n_samp],        box {16}
 };
-
-__device__ __forceinline__ void mbar_init(unsigned long long* bar) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(smem_u32(bar)) : "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(unsigned long long* bar, unsigned bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(bytes)
-                 : "memory");
-}
-__device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned parity) {
-    unsigned done;
-    do {
-        asm volatile(
-            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
-            : "=r"(done)
-            : "r"(smem_u32(bar)), "r"(parity)
-            : "memory");
-    } while (!done);
-}
-__device__ __forceinline__ void tma_1d(void* dst, const CUtensorMap* m, int c0, unsigned long long* bar) {
-    asm volatile(
-        "cp.async.bulk.tensor.1d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2}], [%3];\n" ::"r"(
-            smem_u32(dst)),
-        "l"(m), "r"(c0), "r"(smem_u32(bar))
-        : "memory");
-}
-__device__ __forceinline__ void tma_2d(void* dst, const CUtensorMap* m, int c0, int c1, unsigned long long* bar) {
-    asm volatile(
-        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], "
-        "[%4];\n" ::"r"(smem_u32(dst)),
-        "l"(m), "r"(c0), "r"(c1), "r"(smem_u32(bar))
-        : "memory");
-}
-__device__ __forceinline__ void tma_2d_stream(void* dst, const CUtensorMap* m, int c0, int c1,
-                                              unsigned long long* bar, uint64_t pol) {
-    asm volatile(
-        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1, "
-        "{%2, %3}], [%4], %5;\n" ::"r"(smem_u32(dst)),
-        "l"(m), "r"(c0), "r"(c1), "r"(smem_u32(bar)), "l"(pol)
-        : "memory");
-}
-
-// fp64 / fp32 map reductions (no return value: RED, executed in L2)
-__device__ __forceinline__ void red_f64(double* p, double v) {
-    asm volatile("red.global.add.f64 [%0], %1;" ::"l"(p), "d"(v) : "memory");
-}
-// predicated: no branch around the reduction (the flush stays straight-line code)
-__device__ __forceinline__ void red_f64_if(bool c, double* p, double v) {
-    asm volatile("{\n .reg .pred q;\n setp.ne.u32 q, %2, 0;\n @q red.global.add.f64 [%0], %1;\n}\n" ::"l"(p), "d"(v),
-                 "r"((unsigned)c)
-                 : "memory");
-}
-__device__ __forceinline__ void red_f32(float* p, float v) {
-    asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
-}
 
 // Per-warp shared memory: two staging buffers and the per-sample state (12 KB).  Every TMA
 // destination is 128-byte aligned; the 16 shared-flag bytes of a buffer share their 128-byte slot
@@ -1084,32 +1010,6 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
             if (s_g2l[i] & kHitBit) a.hit_submaps[i] = 1;
     }
 }
-
-// Tensor-map encoder from the driver, fetched through the runtime (no link against libcuda).
-PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
-    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
-    static std::once_flag once;
-    std::call_once(once, [] {
-        void* ptr = nullptr;
-        cudaDriverEntryPointQueryResult q;
-        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &ptr, cudaEnableDefault, &q) == cudaSuccess &&
-            q == cudaDriverEntryPointSuccess)
-            fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(ptr);
-    });
-    return fn;
-}
-
-bool encode_map(CUtensorMap* m, CUtensorMapDataType type, cuuint32_t rank, const void* base, const cuuint64_t* dims,
-                const cuuint64_t* strides, const cuuint32_t* box, CUtensorMapSwizzle swz) {
-    const cuuint32_t es[2] = {1, 1};
-    return tensor_map_encoder()(m, type, rank, const_cast<void*>(base), dims, strides, box, es,
-                                CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_NONE,
-                                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
-}
-
-bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; }
-
-const cuuint64_t kNoStrides[1] = {0};  // rank-1 maps have no strides (a non-null array is passed anyway)
 
 // The TMA path applies when every staged array is 16-byte aligned and rows of the TOD and the
 // det flags are multiples of 16 bytes (n_samp % 16 == 0); otherwise the cp.async path runs (same
