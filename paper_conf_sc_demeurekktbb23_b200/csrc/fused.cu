@@ -314,6 +314,8 @@ struct Slot {
     double r0, r1, r2;  // run sums: sum tod, sum tod cq / r, sum tod sq' / r
     double px, py, ptt; // incremental longitude: projected direction and tt of the previous sample
     P run_key;          // key of the run being aggregated (-1: none)
+    int pk;             // PIPE: key of the finished run flushed at the next sample (-1: none)
+    double pf0, pf1, pf2;  // PIPE: its scaled sums
     int64_t run_elem;   // SCAN: map element of the cached run (-1: none)
     unsigned pend_addr; // SCAN: shared address of the sample whose TOD update is pending (~0: none)
     double pend_c, pend_s;  // SCAN: its eta cal cos / r and 2 eta cal sin' / r
@@ -341,6 +343,8 @@ __device__ __forceinline__ void load_slot(Slot<P>& sl, const FusedArgs& a, int64
     sl.sQ = ok ? scale * sl.etacal : 0.0;
     sl.sU = 2.0 * usign * sl.sQ;
     sl.run_key = -1;
+    sl.pk = -1;
+    sl.pf0 = sl.pf1 = sl.pf2 = 0.0;
     sl.run_elem = -1;
     sl.pend_addr = 0xffffffffu;
     sl.pend_c = sl.pend_s = 0.0;
@@ -526,7 +530,31 @@ __device__ __forceinline__ void flush_lean_pred(bool go, int key, double r0, dou
     }
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool TMA, bool SCAN, bool QUEUE>
+// The lean flush of a PENDING run (the one that ended at the lane's previous sample), written as
+// straight-line predicated code with no memory clobbers: it sits in the same basic block as the
+// next sample's pointing, so the scheduler interleaves the decode / lookup / reduction chain with
+// independent fp64 work instead of running it as a divergent branch (PIPE kernels).
+template <bool NEST, int NNZ, bool OFF>
+__device__ __forceinline__ void flush_pending(int pk, double f0, double f1, double f2, double* __restrict__ zmap,
+                                              int sm_shift, unsigned psm_mask, const HealpixGeom& g,
+                                              uint16_t* g2l) {
+    const bool go = pk >= 0;
+    const unsigned pix = (unsigned)ckey_to_pix_bf<NEST, OFF>(go ? pk : 0, g);
+    const unsigned sm = pix >> sm_shift;
+    const unsigned v = g2l[sm];
+    if (go) g2l[sm] = (uint16_t)(v | kHitBit);
+    const unsigned loc = v & 0x7fffu;
+    if (go && loc != kNoLoc) {
+        double* dst = zmap + (size_t)((loc << sm_shift) + (pix & psm_mask)) * NNZ;
+        atomicAdd(dst, f0);
+        if (NNZ == 3) {
+            atomicAdd(dst + 1, f1);
+            atomicAdd(dst + 2, f2);
+        }
+    }
+}
+
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool TMA, bool SCAN, bool QUEUE, bool PIPE>
 __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
     pointing_to_map_kernel(const Chunk* __restrict__ chunks, int n_chunks, FusedArgs a, HealpixGeom g, KeyConsts kc,
                            unsigned long long* __restrict__ sched, const __grid_constant__ TmaMaps tm) {
@@ -855,7 +883,43 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
             // TOD tile: 1 KB-aligned, row r at r * 128, so the swizzled address of (lane, k) is
             // (tile + row_swz) ^ (8 k): one LOP3 per sample
             const unsigned tile = smem_u32(&ws.tod[p][0][0]) + row_swz;
-            {
+            bool piped = false;
+            if constexpr (PIPE && !SCAN && !DEBUG && !QUEUE && !WIDE) {
+                if (lean) {
+                    // PIPE: the run that ended at sample k-1 is flushed (predicated, branch-free) in
+                    // the same basic block as sample k's pointing, so the two chains interleave
+                    piped = true;
+                    const int kb = cur.k0, ke = cur.k0 + cur.nb;
+                    const unsigned psm_mask = (unsigned)(mg.n_pix_submap - 1);
+#pragma unroll 1
+                    for (int k = kb; k < ke; ++k) {
+                        const bool pixelise = (pmask >> k) & 1u;
+                        const unsigned addr = tile ^ ((unsigned)k << 3);
+                        double x[12];
+                        load_state(k, x);
+                        flush_pending<NEST, NNZ, OFF>(sl.pk, sl.pf0, sl.pf1, sl.pf2, a.zmap, mg.sm_shift, psm_mask, g,
+                                                      cm.g2l);
+                        const StageA o = stage_a<NNZ, HWP, P>(sl, x, kc);
+                        P key = stage_b<NEST, NNZ, WIDE>(o, pixelise, g, kc);
+                        if (!sl.ok) key = -1;
+                        double tod;
+                        asm("ld.shared.f64 %0, [%1];" : "=d"(tod) : "r"(addr));
+                        const bool chg = key != sl.run_key;
+                        sl.pk = chg ? (int)sl.run_key : -1;
+                        sl.pf0 = sl.r0 * sl.sI;
+                        sl.pf1 = sl.r1 * sl.sQ;
+                        sl.pf2 = sl.r2 * sl.sU;
+                        const double t = tod * o.invr;
+                        sl.r0 = (chg ? 0.0 : sl.r0) + tod;
+                        if (NNZ == 3) {
+                            sl.r1 = fma(t, o.cw, chg ? 0.0 : sl.r1);
+                            sl.r2 = fma(t, o.sw, chg ? 0.0 : sl.r2);
+                        }
+                        sl.run_key = key;
+                    }
+                }
+            }
+            if (!piped) {
                 const int kb = cur.k0, ke = cur.k0 + cur.nb;
 #pragma unroll 1
                 for (int k = kb; k < ke; ++k) {
@@ -993,6 +1057,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
                     drain(qn);
                     qn = 0;
                 } else if constexpr (!SCAN) {
+                    if (PIPE && sl.pk >= 0) flush_run((P)sl.pk, sl.pf0, sl.pf1, sl.pf2, sl.det);
                     if (sl.run_key >= 0) flush_run(sl.run_key, sl.r0 * sl.sI, sl.r1 * sl.sQ, sl.r2 * sl.sU, sl.det);
                 }
                 if (nxt.item < 0) break;
@@ -1099,10 +1164,10 @@ void raise_smem_limit(K kern, bool* done_per_dev) {
     }
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool TMA, bool SCAN, bool QUEUE>
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool TMA, bool SCAN, bool QUEUE, bool PIPE>
 cudaError_t launch_k(const WorkList& wl, const FusedArgs& a, const TmaMaps& tm, unsigned long long* sched,
                      cudaStream_t st) {
-    auto kern = pointing_to_map_kernel<NEST, NNZ, HWP, DEBUG, WIDE, TMA, SCAN, QUEUE>;
+    auto kern = pointing_to_map_kernel<NEST, NNZ, HWP, DEBUG, WIDE, TMA, SCAN, QUEUE, PIPE>;
     static bool done[64] = {false};
     raise_smem_limit(kern, done);
     const size_t smem = fused_smem(a);
@@ -1127,15 +1192,15 @@ cudaError_t launch_k(const WorkList& wl, const FusedArgs& a, const TmaMaps& tm, 
     return cudaGetLastError();
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool SCAN, bool QUEUE = false>
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool SCAN, bool QUEUE = false, bool PIPE = false>
 cudaError_t launch_t(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
     TmaMaps tm;
     if (make_tma_maps(a, &tm)) {
         t_fused_path = "tma";
-        return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, true, SCAN, QUEUE>(wl, a, tm, sched, st);
+        return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, true, SCAN, QUEUE, PIPE>(wl, a, tm, sched, st);
     }
     std::memset(&tm, 0, sizeof(tm));
-    return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, false, SCAN, QUEUE>(wl, a, tm, sched, st);
+    return launch_k<NEST, NNZ, HWP, DEBUG, WIDE, false, SCAN, QUEUE, PIPE>(wl, a, tm, sched, st);
 }
 
 // nside <= 4096: 32-bit compact keys; beyond: 64-bit pixel keys
@@ -1146,12 +1211,23 @@ constexpr int64_t kCompactMaxNside = 4096;
 #define TB_QUEUE_MAX_NSIDE 0  // measured r02v: C4 53.5 vs 52.3 ms, C3 0.477 vs 0.467 ms, C2 equal: off
 #endif
 
+// The pipelined predicated flush (PIPE kernels) for nside >= TB_PIPE_MIN_NSIDE, where some lane of
+// a warp ends a run at nearly every sample anyway.
+#ifndef TB_PIPE_MIN_NSIDE
+#define TB_PIPE_MIN_NSIDE 1024  // measured r02p3: C3 0.467 -> 0.442 ms, C4 51.9 -> 49.6 ms; C2 (nside 256) +12 %
+#endif
+
 template <bool NEST, int NNZ, bool HWP, bool DEBUG>
 cudaError_t dispatch_shape(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
     if (a.nside > kCompactMaxNside) return launch_t<NEST, NNZ, HWP, DEBUG, true, false>(wl, a, sched, st);
 #if TB_QUEUE_MAX_NSIDE > 0
     if constexpr (!DEBUG) {
         if (a.nside <= TB_QUEUE_MAX_NSIDE) return launch_t<NEST, NNZ, HWP, false, false, false, true>(wl, a, sched, st);
+    }
+#endif
+#if TB_PIPE_MIN_NSIDE > 0
+    if constexpr (!DEBUG) {
+        if (a.nside >= TB_PIPE_MIN_NSIDE) return launch_t<NEST, NNZ, HWP, false, false, false, false, true>(wl, a, sched, st);
     }
 #endif
     return launch_t<NEST, NNZ, HWP, DEBUG, false, false>(wl, a, sched, st);
