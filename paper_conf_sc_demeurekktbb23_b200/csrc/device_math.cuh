@@ -499,8 +499,8 @@ __device__ __forceinline__ int loc2key32(const HealpixGeom& g, double dz, double
 // is formed once per run, when the run's sum is flushed (ckey_to_pix).  So the per-sample work
 // in the equatorial belt stops at the two floors:
 //   belt: key = (jp << 15) | jm            (jp, jm < 6.9 nside < 2^15)
-//   caps: key = 1 << 30 | payload          NEST: south << 26 | face << 24 | jp << 12 | jm
-//                                          RING: south << 26 | (north pixel, or npix - 1 - pixel)
+//   caps: NEST: the cap pixel re-expressed as a belt key (one decoder for both, see loc2ckey)
+//         RING: key = 1 << 30 | south << 26 | (north pixel, or npix - 1 - pixel)
 // Any two different pixels get different keys; one pixel can get two keys (the unwrapped
 // longitude of the incremental chain, OFF below, reaches a pixel from tt and tt + 4), which
 // only splits a run.  Keys are non-negative; -1 means "no pixel".
@@ -575,7 +575,16 @@ __device__ __forceinline__ int loc2ckey(const HealpixGeom& g, const KeyConsts& k
         int jm = floor_nonneg(__dmul_rn(__dsub_rn(1.0, tp), tmp));
         jp = min(jp, m);
         jm = min(jm, m);
-        return kCapBit | (south << 26) | (face << 24) | (jp << 12) | jm;
+        // the cap pixel (face F or F + 8, ix, iy) written in the BELT key format, so one decoder
+        // serves both (ckey_to_pix): the belt decode gives face = (min(ifp, ifm) (+3 OFF) mod 4)
+        // + 4 (1 + ifp - ifm), ix = jm mod N, iy = N - 1 - (jp mod N).  North (ix, iy) = (N-1-jm,
+        // N-1-jp): ifp = F + d, ifm = F + 1 + d; south (ix, iy) = (jp, jm): ifm = F + d,
+        // ifp = F + 1 + d (d = 1 when OFF).  ifp, ifm <= 5, so the fields stay below 6 N < 2^15.
+        constexpr int d = OFF ? 1 : 0;
+        const int lo = (face + d) << g.order, hi = (face + 1 + d) << g.order;
+        const int kp = south ? (hi | (m - jm)) : (lo | jp);
+        const int km = south ? (lo | jp) : (hi | (m - jm));
+        return (kp << 15) | km;
     }
 }
 
@@ -584,17 +593,10 @@ template <bool NEST, bool OFF>
 __device__ __forceinline__ int ckey_to_pix(int key, const HealpixGeom& g) {
     const int nside = (int)g.nside;
     const int m = nside - 1;
-    if (key & kCapBit) {
+    if (!NEST && (key & kCapBit)) {  // RING caps (NEST cap keys are in the belt format)
         const int south = (key >> 26) & 1;
-        if (!NEST) {
-            const int p = key & ((1 << 26) - 1);
-            return south ? (int)g.npix - 1 - p : p;
-        }
-        const int face = ((key >> 24) & 3) + 8 * south;
-        const int jp = (key >> 12) & 0xfff, jm = key & 0xfff;
-        const int ix = south ? jp : m - jm;
-        const int iy = south ? jm : m - jp;
-        return face * (nside * nside) + (int)interleave16((uint32_t)ix, (uint32_t)iy);
+        const int p = key & ((1 << 26) - 1);
+        return south ? (int)g.npix - 1 - p : p;
     }
     const int jp = key >> 15, jm = key & 0x7fff;
     if (!NEST) {
@@ -620,9 +622,9 @@ template <bool NEST, bool OFF>
 __device__ __forceinline__ int ckey_to_pix_bf(int key, const HealpixGeom& g) {
     const int nside = (int)g.nside;
     const int m = nside - 1;
-    const bool cap = key & kCapBit;
-    const int south = (key >> 26) & 1;
     if (!NEST) {
+        const bool cap = key & kCapBit;
+        const int south = (key >> 26) & 1;
         const int nl4 = 4 * nside;
         const int jp = key >> 15, jm = key & 0x7fff;
         const int ir = nside + 1 + jp - jm;
@@ -633,21 +635,12 @@ __device__ __forceinline__ int ckey_to_pix_bf(int key, const HealpixGeom& g) {
         const int capp = south ? (int)g.npix - 1 - p : p;
         return cap ? capp : belt;
     }
-    // belt
-    const int bjp = (key >> 15) & 0x7fff, bjm = key & 0x7fff;
-    const int ifp = bjp >> g.order, ifm = bjm >> g.order;
+    // NEST: one decoder (cap keys are in the belt format, see loc2ckey)
+    const int jp = key >> 15, jm = key & 0x7fff;
+    const int ifp = jp >> g.order, ifm = jm >> g.order;
     const int fmin = (ifp < ifm ? ifp : ifm) + (OFF ? 3 : 0);
-    const int bface = (fmin & 3) + 4 * (1 + ifp - ifm);
-    const int bix = bjm & m, biy = (bjp & m) ^ m;
-    // cap
-    const int cjp = (key >> 12) & 0xfff, cjm = key & 0xfff;
-    const int cface = ((key >> 24) & 3) + 8 * south;
-    const int cix = south ? cjp : m - cjm;
-    const int ciy = south ? cjm : m - cjp;
-    const int face = cap ? cface : bface;
-    const int ix = cap ? cix : bix;
-    const int iy = cap ? ciy : biy;
-    return face * (nside * nside) + (int)interleave16((uint32_t)ix, (uint32_t)iy);
+    const int face = (fmin & 3) + 4 * (1 + ifp - ifm);
+    return face * (nside * nside) + (int)interleave16((uint32_t)(jm & m), (uint32_t)((jp & m) ^ m));
 }
 
 // Pixel of a run key (see loc2key32).

@@ -363,9 +363,10 @@ struct StageA {
 };
 
 // (2/pi) atan(t) = t Q(t^2) for |t| <= kIncrMax = 0.01 (TB_INCR_MAX, in the constant bank): the
-// Taylor series to t^7; the first omitted term is (2/pi) t^9 / 9 <= 7e-20 (absolute) at |t| = 0.01.
-__constant__ double kIncrQ[4] = {0.63661977236758134308, -0.21220659078919378103, 0.12732395447351626862,
-                                 -0.090945681766797334729};
+// Taylor series to t^5; the omitted tail is below (2/pi) t^7 / 7 <= 9.1e-16 quarter turns per step
+// at |t| = 0.01, so a chain of <= 127 steps drifts by < 1.2e-13 quarter turns (1.8e-13 rad), inside
+// rule T1's 1e-12 rad.
+__constant__ double kIncrQ[3] = {0.63661977236758134308, -0.21220659078919378103, 0.12732395447351626862};
 
 // OFF: 32-bit keys with the incremental longitude carried as tt + 1 WITHOUT wrapping (see below).
 template <int NNZ, typename P>
@@ -403,22 +404,18 @@ __device__ __forceinline__ StageA stage_a(Slot<P>& sl, const double* x, const Ke
         // the belt floors need N (tt + 1/2) - 1/2 = N t q + (N ptt + N/2 - 1/2): the second term is
         // formed while the reciprocal is in flight, so the key path after t is short (Estrin
         // form of q: depth 2 instead of 3)
-        const double pre = fma(kc.dn, sl.ptt, kc.dn_half_m);
         {
             const double t = cr * inv;
             o.invr = dot * inv;
             const double s2 = t * t;
-            const double nt = kc.dn * t;  // exact (power-of-two scale)
-            const double qa = fma(kIncrQ[1], s2, kIncrQ[0]);
-            const double qb = fma(kIncrQ[3], s2, kIncrQ[2]);
-            const double q = fma(s2 * s2, qb, qa);
+            const double q = fma(fma(kIncrQ[2], s2, kIncrQ[1]), s2, kIncrQ[0]);
             double tt = fma(t, q, sl.ptt);
             if constexpr (!OFF) {
                 if (__double2hiint(tt) < 0) tt += 4.0;
                 if (__double2hiint(tt) >= 0x40100000) tt -= 4.0;
             }
             o.tt = tt;
-            o.t1m = fma(nt, q, pre);
+            o.t1m = fma(kc.dn, tt, kc.dn_half_m);  // N (tt + 1/2) - 1/2 (N tt exact)
         }
         // |cross| < kIncrMax dot  <=>  dot > 0 and |t| < kIncrMax; false at dot = 0 and for steps
         // beyond a quarter turn
@@ -891,26 +888,26 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
                     piped = true;
                     const int kb = cur.k0, ke = cur.k0 + cur.nb;
                     const unsigned psm_mask = (unsigned)(mg.n_pix_submap - 1);
+                    const unsigned pm = sl.ok ? pmask : 0u;  // a lane without a detector: key -1
 #pragma unroll 1
                     for (int k = kb; k < ke; ++k) {
-                        const bool pixelise = (pmask >> k) & 1u;
+                        const bool pixelise = (pm >> k) & 1u;
                         const unsigned addr = tile ^ ((unsigned)k << 3);
                         double x[12];
                         load_state(k, x);
                         flush_pending<NEST, NNZ, OFF>(sl.pk, sl.pf0, sl.pf1, sl.pf2, a.zmap, mg.sm_shift, psm_mask, g,
                                                       cm.g2l);
                         const StageA o = stage_a<NNZ, HWP, P>(sl, x, kc);
-                        P key = stage_b<NEST, NNZ, WIDE>(o, pixelise, g, kc);
-                        if (!sl.ok) key = -1;
+                        const P key = stage_b<NEST, NNZ, WIDE>(o, pixelise, g, kc);
                         double tod;
                         asm("ld.shared.f64 %0, [%1];" : "=d"(tod) : "r"(addr));
                         const bool chg = key != sl.run_key;
                         sl.pk = chg ? (int)sl.run_key : -1;
-                        sl.pf0 = sl.r0 * sl.sI;
+                        sl.pf0 = sl.r0;
                         sl.pf1 = sl.r1 * sl.sQ;
                         sl.pf2 = sl.r2 * sl.sU;
                         const double t = tod * o.invr;
-                        sl.r0 = (chg ? 0.0 : sl.r0) + tod;
+                        sl.r0 = fma(tod, sl.sI, chg ? 0.0 : sl.r0);
                         if (NNZ == 3) {
                             sl.r1 = fma(t, o.cw, chg ? 0.0 : sl.r1);
                             sl.r2 = fma(t, o.sw, chg ? 0.0 : sl.r2);
@@ -998,7 +995,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
                         // reset once, before the flush, so the compiler keeps one copy of it)
                         if constexpr (QUEUE) {
                             const bool chg = key != sl.run_key;
-                            push(chg && sl.run_key >= 0, sl.run_key, sl.r0 * sl.sI, sl.r1 * sl.sQ, sl.r2 * sl.sU);
+                            push(chg && sl.run_key >= 0, sl.run_key, sl.r0, sl.r1 * sl.sQ, sl.r2 * sl.sU);
                             if (chg) {
                                 sl.run_key = key;
                                 sl.r0 = sl.r1 = sl.r2 = 0.0;
@@ -1007,7 +1004,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
                         } else if (lean) {
                             // straight-line flush (see flush_lean_pred)
                             const bool chg = key != sl.run_key;
-                            const double f0 = sl.r0 * sl.sI, f1 = sl.r1 * sl.sQ, f2 = sl.r2 * sl.sU;
+                            const double f0 = sl.r0, f1 = sl.r1 * sl.sQ, f2 = sl.r2 * sl.sU;
                             flush_lean_pred<NEST, NNZ, OFF>(chg && sl.run_key >= 0, (int)sl.run_key, f0, f1, f2, a, g,
                                                             cm.g2l);
                             const double keepr = chg ? 0.0 : 1.0;
@@ -1018,12 +1015,12 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
 #endif
                         } else if (key != sl.run_key) {
                             const P old = sl.run_key;
-                            const double f0 = sl.r0 * sl.sI, f1 = sl.r1 * sl.sQ, f2 = sl.r2 * sl.sU;
+                            const double f0 = sl.r0, f1 = sl.r1 * sl.sQ, f2 = sl.r2 * sl.sU;
                             sl.run_key = key;
                             sl.r0 = sl.r1 = sl.r2 = 0.0;
                             if (old >= 0) flush_run(old, f0, f1, f2, sl.det);
                         }
-                        sl.r0 += tod;
+                        sl.r0 = fma(tod, sl.sI, sl.r0);
                         if (NNZ == 3) {
                             const double t = tod * o.invr;
                             sl.r1 = fma(t, o.cw, sl.r1);
@@ -1053,12 +1050,12 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
 
             if (nxt.item != cur.item) {
                 if constexpr (QUEUE) {
-                    push(sl.run_key >= 0, sl.run_key, sl.r0 * sl.sI, sl.r1 * sl.sQ, sl.r2 * sl.sU);  // open runs
+                    push(sl.run_key >= 0, sl.run_key, sl.r0, sl.r1 * sl.sQ, sl.r2 * sl.sU);  // open runs
                     drain(qn);
                     qn = 0;
                 } else if constexpr (!SCAN) {
                     if (PIPE && sl.pk >= 0) flush_run((P)sl.pk, sl.pf0, sl.pf1, sl.pf2, sl.det);
-                    if (sl.run_key >= 0) flush_run(sl.run_key, sl.r0 * sl.sI, sl.r1 * sl.sQ, sl.r2 * sl.sU, sl.det);
+                    if (sl.run_key >= 0) flush_run(sl.run_key, sl.r0, sl.r1 * sl.sQ, sl.r2 * sl.sU, sl.det);
                 }
                 if (nxt.item < 0) break;
                 load_slot<P>(sl, a, nxt.d0 + lane, lane < nxt.nrows, nxt.d0);
