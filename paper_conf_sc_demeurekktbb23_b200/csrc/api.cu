@@ -210,7 +210,10 @@ int fused_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, int64_
     const int64_t groups = (n_det + 31) / 32, warps = (int64_t)num_sms() * 16, want = 4 * warps;
     // large focal planes (>= 64 detector groups: C4, C5) take 64-sample chunks: the warps in flight
     // then span half the time window, so the map lines they scatter into are reused more in L2
-    int chunk = groups >= 64 ? kFusedChunk / 2 : kFusedChunk;
+#ifndef TB_LARGE_FP_CHUNK
+#define TB_LARGE_FP_CHUNK (kFusedChunk / 2)
+#endif
+    int chunk = groups >= 64 ? TB_LARGE_FP_CHUNK : kFusedChunk;
     while (chunk > 16 && (n_samples / chunk) * groups < want) chunk /= 2;
 #ifndef TB_NO_TAIL
     const int64_t tail =
