@@ -201,19 +201,18 @@ int get_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, cudaStre
 // so that there are at least ~4 items per resident warp.  Items are handed out in list order,
 // so the LAST items set the kernel's tail: the last TB_TAIL_ITEMS items' worth of samples per
 // resident warp are cut into kTailChunk-sample chunks.  Only the final list is built and cached.
-int fused_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, int64_t n_det, cudaStream_t st,
-                   WorkListLease* out) {
+int fused_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, int64_t n_det, int64_t nside,
+                   cudaStream_t st, WorkListLease* out) {
     int rc = validate_intervals(iv, n, n_samp);
     if (rc != TOAST_OK) return rc;
     int64_t n_samples = 0;
     for (int64_t i = 0; i < n; ++i) n_samples += iv[i].last - iv[i].first + 1;
     const int64_t groups = (n_det + 31) / 32, warps = (int64_t)num_sms() * 16, want = 4 * warps;
-    // large focal planes (>= 64 detector groups: C4, C5) take 64-sample chunks: the warps in flight
-    // then span half the time window, so the map lines they scatter into are reused more in L2
-#ifndef TB_LARGE_FP_CHUNK
-#define TB_LARGE_FP_CHUNK (kFusedChunk / 2)
-#endif
-    int chunk = groups >= 64 ? TB_LARGE_FP_CHUNK : kFusedChunk;
+    // large focal planes (>= 64 detector groups) on fine maps (nside >= 4096: C5) take 64-sample
+    // chunks: the warps in flight then span half the time window, so the map lines they scatter
+    // into are reused more in L2 (C5 2.57 -> 2.46 ms); at nside 2048 (C4) the longer chunks win
+    // (fewer item switches and full-arctangent restarts: C4 46.4 -> 45.6 ms, r02p8)
+    int chunk = (groups >= 64 && nside >= 4096) ? kFusedChunk / 2 : kFusedChunk;
     while (chunk > 16 && (n_samples / chunk) * groups < want) chunk /= 2;
 #ifndef TB_NO_TAIL
     const int64_t tail =
@@ -493,7 +492,7 @@ int toast_pointing_to_map_ex(const double* fp_quats, const double* boresight, co
     if (opts && opts->map_f32 && (pixels_out || weights_out))
         return fail(TOAST_EINVAL, "debug outputs are not available with an fp32 map");
     WorkListLease lease;
-    rc = fused_worklist(intervals, n_intervals, n_samp, n_det, (cudaStream_t)stream, &lease);
+    rc = fused_worklist(intervals, n_intervals, n_samp, n_det, nside, (cudaStream_t)stream, &lease);
     if (rc != TOAST_OK) return rc;
     if ((int64_t)lease.wl.n_chunks * ((n_det + 31) / 32) >= (int64_t(1) << 31))
         return fail(TOAST_EUNSUPPORTED, "more than 2^31 work items (split the call over detectors)");
@@ -575,7 +574,7 @@ extern "C" int toast_pointing_to_tod_ex(const double* fp_quats, const double* bo
     }
     if (opts && opts->dropped) return fail(TOAST_EINVAL, "the dropped-sample counter applies to pointing_to_map only");
     WorkListLease lease;
-    rc = fused_worklist(intervals, n_intervals, n_samp, n_det, (cudaStream_t)stream, &lease);
+    rc = fused_worklist(intervals, n_intervals, n_samp, n_det, nside, (cudaStream_t)stream, &lease);
     if (rc != TOAST_OK) return rc;
     if ((int64_t)lease.wl.n_chunks * ((n_det + 31) / 32) >= (int64_t(1) << 31))
         return fail(TOAST_EUNSUPPORTED, "more than 2^31 work items (split the call over detectors)");

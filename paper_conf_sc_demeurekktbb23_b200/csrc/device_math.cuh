@@ -512,34 +512,34 @@ constexpr int kCapBit = 1 << 30;
 // textbook expression (reading S6) only when the argument lies within ~2 ulp of an integer, i.e.
 // for directions within ~1e-15 rad of a pixel boundary (rule T1 allows 1e-12 rad).
 struct KeyConsts {
-    double dn, dn_half_m, dn_3q;  // N, N/2 - 1/2, 3N/4 (exact)
+    double dn, dn_half, dn_3q;  // N, N/2, 3N/4 (exact)
 };
 inline KeyConsts make_key_consts(int64_t nside) {
     KeyConsts k;
     k.dn = (double)nside;
-    k.dn_half_m = 0.5 * (double)nside - 0.5;
+    k.dn_half = 0.5 * (double)nside;
     k.dn_3q = 0.75 * (double)nside;
     return k;
 }
 
-// floor(x + 1/2) - ... : the belt floors as ROUND-TO-NEAREST of (argument - 1/2) on the fp64 pipe:
-// adding 1.5 2^52 rounds to an integer held in the low word (two fp64 adds of latency instead of
-// the ~34-cycle F2I.F64, measured on B200: scripts/fp64_microbench.cu).  It equals floor(argument)
-// except when the argument is within an ulp or so of an integer (ties, and the one rounding of the
-// shifted argument), i.e. for directions within ~1e-15 rad of a pixel boundary (rule T1).
-__device__ __forceinline__ int round_shifted(double x_minus_half) {
-    return __double2loint(x_minus_half + 6755399441055744.0);
+// floor(x) for -2^31 <= x < 2^31 on the fp64 adder: x + 1.5 2^52 rounded toward -infinity is the
+// integer 1.5 2^52 + floor(x), held in the low word (one DADD.RM of ~9 cycles instead of the
+// ~34-cycle F2I.F64, measured on B200: scripts/fp64_microbench.cu).  Exact: it equals the F2I floor
+// of the same double for every x >= 0.
+__device__ __forceinline__ int floor_rd(double x) {
+    return __double2loint(__dadd_rd(x, 6755399441055744.0));
 }
+__device__ __forceinline__ double floor_rd_value(double big) { return big - 6755399441055744.0; }
 
 template <bool NEST, bool OFF>
-__device__ __forceinline__ int loc2ckey(const HealpixGeom& g, const KeyConsts& kc, double dz, double tt, double t1m,
+__device__ __forceinline__ int loc2ckey(const HealpixGeom& g, const KeyConsts& kc, double dz, double tt, double t1,
                                         double dx, double dy) {
     const double za = fabs(dz);
     // the belt key is formed unconditionally (straight-line, so the scheduler can overlap it with
     // independent work); only the caps branch.
-    // t1m = N (tt + 1/2) - 1/2;  jp = floor(N (tt + 1/2) - 3N/4 z), jm = floor(... + 3N/4 z)
-    const int bjp = round_shifted(fma(-dz, kc.dn_3q, t1m));
-    const int bjm = round_shifted(fma(dz, kc.dn_3q, t1m));
+    // t1 = N (tt + 1/2);  jp = floor(N (tt + 1/2) - 3N/4 z), jm = floor(... + 3N/4 z)
+    const int bjp = floor_rd(fma(-dz, kc.dn_3q, t1));
+    const int bjm = floor_rd(fma(dz, kc.dn_3q, t1));
     const int belt = (bjp << 15) | bjm;
     if (za <= TB_TWO_THIRD) return belt;
     const int nside = (int)g.nside;
@@ -553,11 +553,13 @@ __device__ __forceinline__ int loc2ckey(const HealpixGeom& g, const KeyConsts& k
     }
     const int south = dz < 0.0 ? 1 : 0;
     if (!NEST) {
-        const double tp = __dsub_rn(tt, small_int_to_double(floor_nonneg(tt)));
-        const int jp = floor_nonneg(__dmul_rn(tp, tmp));
-        const int jm = floor_nonneg(__dmul_rn(__dsub_rn(1.0, tp), tmp));
+        // the cap floors on the fp64 adder (floor_rd: bit-identical to the F2I floors of the same
+        // products, ~25 cycles shorter each)
+        const double tp = __dsub_rn(tt, floor_rd_value(__dadd_rd(tt, 6755399441055744.0)));
+        const int jp = floor_rd(__dmul_rn(tp, tmp));
+        const int jm = floor_rd(__dmul_rn(__dsub_rn(1.0, tp), tmp));
         const int ir = jp + jm + 1;
-        int ip = floor_nonneg(__dmul_rn(tt, small_int_to_double(ir)));
+        int ip = floor_rd(__dmul_rn(tt, small_int_to_double(ir)));
         if (OFF) {
             ip -= ir;  // in [-0.82 ir, 4.82 ir)
             if (ip < 0) ip += 4 * ir;
@@ -567,12 +569,17 @@ __device__ __forceinline__ int loc2ckey(const HealpixGeom& g, const KeyConsts& k
         const int p = south ? 2 * ir * (ir + 1) - 1 - ip : 2 * ir * (ir - 1) + ip;
         return kCapBit | (south << 26) | p;
     } else {
-        int ntt = floor_nonneg(tt);
-        if (!OFF && ntt > 3) ntt = 3;
-        const double tp = __dsub_rn(tt, small_int_to_double(ntt));
+        const double bt = __dadd_rd(tt, 6755399441055744.0);
+        int ntt = __double2loint(bt);
+        double dntt = floor_rd_value(bt);
+        if (!OFF && ntt > 3) {
+            ntt = 3;
+            dntt = 3.0;
+        }
+        const double tp = __dsub_rn(tt, dntt);
         const int face = OFF ? ((ntt + 3) & 3) : ntt;
-        int jp = floor_nonneg(__dmul_rn(tp, tmp));
-        int jm = floor_nonneg(__dmul_rn(__dsub_rn(1.0, tp), tmp));
+        int jp = floor_rd(__dmul_rn(tp, tmp));
+        int jm = floor_rd(__dmul_rn(__dsub_rn(1.0, tp), tmp));
         jp = min(jp, m);
         jm = min(jm, m);
         // the cap pixel (face F or F + 8, ix, iy) written in the BELT key format, so one decoder

@@ -363,7 +363,7 @@ __device__ __forceinline__ void load_slot(Slot<P>& sl, const FusedArgs& a, int64
 struct StageA {
     double dx, dy, dz, tt;
     double cw, sw, invr;  // r cos 2(psi + 2 chi), r sin 2(psi + 2 chi) / 2, 1/r
-    double t1m;           // N (tt + 1/2) - 1/2: the belt floors' common term (see loc2ckey_t1m)
+    double t1m;           // N (tt + 1/2): the belt floors' common term (see loc2ckey)
 };
 
 // (2/pi) atan(t) = t Q(t^2) for |t| <= kIncrMax = 0.01 (TB_INCR_MAX, in the constant bank): the
@@ -419,7 +419,7 @@ __device__ __forceinline__ StageA stage_a(Slot<P>& sl, const double* x, const Ke
                 if (__double2hiint(tt) >= 0x40100000) tt -= 4.0;
             }
             o.tt = tt;
-            o.t1m = fma(kc.dn, tt, kc.dn_half_m);  // N (tt + 1/2) - 1/2 (N tt exact)
+            o.t1m = fma(kc.dn, tt, kc.dn_half);  // N (tt + 1/2) (N tt exact)
         }
         // |cross| < kIncrMax dot  <=>  dot > 0 and |t| < kIncrMax; false at dot = 0 and for steps
         // beyond a quarter turn
@@ -429,7 +429,7 @@ __device__ __forceinline__ StageA stage_a(Slot<P>& sl, const double* x, const Ke
             // so it stays in (0.18, 5.82); loc2ckey<NEST, true> folds it back
             double A, B;
             o.tt = lon_pol_raw(o.dx, o.dy, bx, by, A, B, o.invr) + (OFF ? 1.0 : 0.0);
-            o.t1m = fma(kc.dn, o.tt, kc.dn_half_m);
+            o.t1m = fma(kc.dn, o.tt, kc.dn_half);
         }
         sl.px = o.dx;
         sl.py = o.dy;
@@ -444,7 +444,7 @@ __device__ __forceinline__ StageA stage_a(Slot<P>& sl, const double* x, const Ke
         }
     } else {
         o.tt = quarter_turns(o.dx, o.dy);
-        o.t1m = fma(kc.dn, o.tt, kc.dn_half_m);
+        o.t1m = fma(kc.dn, o.tt, kc.dn_half);
     }
     return o;
 }
