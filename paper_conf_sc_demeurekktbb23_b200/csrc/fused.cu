@@ -555,7 +555,7 @@ __device__ __forceinline__ void flush_pending(int pk, double f0, double f1, doub
     }
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool TMA, bool SCAN, bool QUEUE, bool PIPE>
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool TMA, bool SCAN, bool QUEUE, int PIPE>
 __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
     pointing_to_map_kernel(const Chunk* __restrict__ chunks, int n_chunks, FusedArgs a, HealpixGeom g, KeyConsts kc,
                            unsigned long long* __restrict__ sched, const __grid_constant__ TmaMaps tm) {
@@ -889,7 +889,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
             // (tile + row_swz) ^ (8 k): one LOP3 per sample
             const unsigned tile = smem_u32(&ws.tod[p][0][0]) + row_swz;
             bool piped = false;
-            if constexpr (PIPE && !SCAN && !DEBUG && !QUEUE && !WIDE) {
+            if constexpr (PIPE != 0 && !SCAN && !DEBUG && !QUEUE && !WIDE) {
                 if (lean) {
                     // PIPE: the run that ended at sample k-1 is flushed (predicated, branch-free) in
                     // the same basic block as sample k's pointing, so the two chains interleave
@@ -903,9 +903,22 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
                         const unsigned addr = tile ^ ((unsigned)k << 3);
                         double x[12];
                         load_state(k, x);
-                        flush_pending<NEST, NNZ, OFF>(sl.pk, sl.pf0, sl.pf1, sl.pf2, a.zmap, mg.sm_shift, psm_mask, g,
-                                                      cm.g2l);
-                        const StageA o = stage_a<NNZ, HWP, P>(sl, x, kc);
+                        StageA o;
+                        if constexpr (PIPE == 2) {
+                            // hybrid (nside < 1024, where most samples end no run): the interleaved
+                            // flush + pointing block only when some lane has a pending run
+                            if (__any_sync(kFull, sl.pk >= 0)) {
+                                flush_pending<NEST, NNZ, OFF>(sl.pk, sl.pf0, sl.pf1, sl.pf2, a.zmap, mg.sm_shift,
+                                                              psm_mask, g, cm.g2l);
+                                o = stage_a<NNZ, HWP, P>(sl, x, kc);
+                            } else {
+                                o = stage_a<NNZ, HWP, P>(sl, x, kc);
+                            }
+                        } else {
+                            flush_pending<NEST, NNZ, OFF>(sl.pk, sl.pf0, sl.pf1, sl.pf2, a.zmap, mg.sm_shift, psm_mask,
+                                                          g, cm.g2l);
+                            o = stage_a<NNZ, HWP, P>(sl, x, kc);
+                        }
                         P key;
                         if constexpr (HWP && NNZ == 3) {
                             key = stage_b<NEST, NNZ, WIDE>(o, (pm >> k) & 1u, g, kc);
@@ -1067,7 +1080,7 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
                     drain(qn);
                     qn = 0;
                 } else if constexpr (!SCAN) {
-                    if (PIPE && sl.pk >= 0) flush_run((P)sl.pk, sl.pf0, sl.pf1, sl.pf2, sl.det);
+                    if (PIPE != 0 && sl.pk >= 0) flush_run((P)sl.pk, sl.pf0, sl.pf1, sl.pf2, sl.det);
                     if (sl.run_key >= 0) flush_run(sl.run_key, sl.r0, sl.r1 * sl.sQ, sl.r2 * sl.sU, sl.det);
                 }
                 if (nxt.item < 0) break;
@@ -1174,7 +1187,7 @@ void raise_smem_limit(K kern, bool* done_per_dev) {
     }
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool TMA, bool SCAN, bool QUEUE, bool PIPE>
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool TMA, bool SCAN, bool QUEUE, int PIPE>
 cudaError_t launch_k(const WorkList& wl, const FusedArgs& a, const TmaMaps& tm, unsigned long long* sched,
                      cudaStream_t st) {
     auto kern = pointing_to_map_kernel<NEST, NNZ, HWP, DEBUG, WIDE, TMA, SCAN, QUEUE, PIPE>;
@@ -1202,7 +1215,7 @@ cudaError_t launch_k(const WorkList& wl, const FusedArgs& a, const TmaMaps& tm, 
     return cudaGetLastError();
 }
 
-template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool SCAN, bool QUEUE = false, bool PIPE = false>
+template <bool NEST, int NNZ, bool HWP, bool DEBUG, bool WIDE, bool SCAN, bool QUEUE = false, int PIPE = 0>
 cudaError_t launch_t(const WorkList& wl, const FusedArgs& a, unsigned long long* sched, cudaStream_t st) {
     TmaMaps tm;
     if (make_tma_maps(a, &tm)) {
@@ -1223,6 +1236,9 @@ constexpr int64_t kCompactMaxNside = 4096;
 
 // The pipelined predicated flush (PIPE kernels) for nside >= TB_PIPE_MIN_NSIDE, where some lane of
 // a warp ends a run at nearly every sample anyway.
+#ifndef TB_PIPE_HYB
+#define TB_PIPE_HYB 1  // below TB_PIPE_MIN_NSIDE: the hybrid PIPE loop (measured r02p9: C2 0.462 -> 0.451 ms; C3 +3.6 %, C4 +4.3 % with it)
+#endif
 #ifndef TB_PIPE_MIN_NSIDE
 #define TB_PIPE_MIN_NSIDE 1024  // measured r02p3: C3 0.467 -> 0.442 ms, C4 51.9 -> 49.6 ms; C2 (nside 256) +12 %
 #endif
@@ -1237,7 +1253,10 @@ cudaError_t dispatch_shape(const WorkList& wl, const FusedArgs& a, unsigned long
 #endif
 #if TB_PIPE_MIN_NSIDE > 0
     if constexpr (!DEBUG) {
-        if (a.nside >= TB_PIPE_MIN_NSIDE) return launch_t<NEST, NNZ, HWP, false, false, false, false, true>(wl, a, sched, st);
+        if (a.nside >= TB_PIPE_MIN_NSIDE) return launch_t<NEST, NNZ, HWP, false, false, false, false, 1>(wl, a, sched, st);
+#if TB_PIPE_HYB
+        return launch_t<NEST, NNZ, HWP, false, false, false, false, 2>(wl, a, sched, st);
+#endif
     }
 #endif
     return launch_t<NEST, NNZ, HWP, DEBUG, false, false>(wl, a, sched, st);
