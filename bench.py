@@ -78,7 +78,7 @@ def parse():
     ap.add_argument("--graph", type=int, default=0,
                     help="launch-bound configs (C1, SURVEY 8(d)): one step = a CUDA graph of G back-to-back "
                          "(zero map + fused call)s, captured once and replayed")
-    ap.add_argument("--reduce", default="auto", choices=["auto", "dense", "packed", "scatter"],
+    ap.add_argument("--reduce", default="auto", choices=["auto", "dense", "packed", "scatter", "nvls"],
                     help="N>1 map reduction: dense all_reduce, all_reduce of the union of hit submaps (packed), "
                          "or the sparse distributed map domain (compact map + reduce_scatter, SURVEY 8(f) f3)")
     return ap.parse_args()
@@ -351,7 +351,10 @@ def main():
         raws = [tuple(list(r[:19]) + [hits.data_ptr()] + list(r[20:])) for r in raws]
         torch.cuda.synchronize()
 
-    packed = own is None and world > 1 and (args.reduce == "packed" or (args.reduce == "auto" and zmap.numel() * 8 > (256 << 20)))
+    packed = own is None and world > 1 and (args.reduce in ("packed", "nvls") or
+                                            (args.reduce == "auto" and zmap.numel() * 8 > (256 << 20)))
+    # --reduce nvls: the packed union summed in the switch by toast_map_allreduce_nvls (f3)
+    nvls_red = tdist.NvlsReducer(zmap.numel(), dev) if (world > 1 and args.reduce == "nvls") else None
     reduced = {"bytes": 0}
     kern_events = []  # (start, end) of every fused map launch in the timed region
 
@@ -380,7 +383,7 @@ def main():
                 _, reduced["bytes"] = tdist.reduce_scatter_map(zmap, own)
             elif packed:
                 tdist.union_hit_submaps(hits)
-                _, reduced["bytes"] = tdist.reduce_map(zmap, hit_submaps=hits, global2local=g2l)
+                _, reduced["bytes"] = tdist.reduce_map(zmap, hit_submaps=hits, global2local=g2l, nvls=nvls_red)
             else:
                 _, reduced["bytes"] = tdist.reduce_map(zmap)
 
@@ -431,7 +434,7 @@ def main():
             tdist.reduce_scatter_map(zmap, own)
         elif packed:
             tdist.union_hit_submaps(hits)
-            tdist.reduce_map(zmap, hit_submaps=hits, global2local=g2l)
+            tdist.reduce_map(zmap, hit_submaps=hits, global2local=g2l, nvls=nvls_red)
         else:
             tdist.reduce_map(zmap)
         b.record(stream)
@@ -478,7 +481,7 @@ def main():
     e2e = None
     if not args.no_e2e:
         e2e = run_e2e(args, obs, zmap, hits, g2l, world, stream, packed,
-                      total_det_samples / (args.graph if graph is not None else 1), scan_map_in, own)
+                      total_det_samples / (args.graph if graph is not None else 1), scan_map_in, own, nvls_red)
 
     # ---- roofline of the dominant kernel (the fused pointing->map kernel), per launch
     det_per_launch = det_samples / len(obs) / (args.graph if graph is not None else 1)
@@ -536,8 +539,10 @@ def main():
                                  (sum(o.w.n_det * o.w.n_samp * 8 for o in obs) / 1e6),
                            "parallelism": (f"dp{world}: " + ("detector blocks of one observation" if shard == "det"
                                                              else "one observation per rank") +
-                                           " + NCCL " + ("packed all_reduce (union of hit submaps)" if packed
-                                                         else "all_reduce") + " of the map") if world > 1
+                                           (" + NVLS multimem all-reduce (toast_map_allreduce_nvls) of the union of "
+                                            "hit submaps" if nvls_red is not None else
+                                            " + NCCL " + ("packed all_reduce (union of hit submaps)" if packed
+                                                          else "all_reduce") + " of the map")) if world > 1
                            else "single GPU",
                            "step": "zero map + " + ("(pointing_to_tod + pointing_to_map) per observation"
                                                     if scan_map_in is not None else "toast_pointing_to_map") +
@@ -562,7 +567,8 @@ def main():
         dist.destroy_process_group()
 
 
-def run_e2e(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples, with_scan, own=None):
+def run_e2e(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples, with_scan, own=None,
+            nvls_red=None):
     """Same metric through the public API with host buffers: every step copies the step's inputs
     from pinned host memory (the TOD in 256-detector blocks through two device staging buffers,
     overlapped with the fused kernel: streaming.Streamer) and reads the map back."""
@@ -571,7 +577,8 @@ def run_e2e(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples
     from paper_conf_sc_demeurekktbb23_b200 import dist as tdist
     from paper_conf_sc_demeurekktbb23_b200.streaming import HostInputs, Streamer
     if with_scan is not None:
-        return run_e2e_round_trip(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples, own, with_scan)
+        return run_e2e_round_trip(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples, own, with_scan,
+                                  nvls_red)
     hosts, streamers = [], []
     try:
         for o in obs:
@@ -606,7 +613,7 @@ def run_e2e(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples
                 tdist.reduce_scatter_map(zmap, own)
             elif packed:
                 tdist.union_hit_submaps(hits)
-                tdist.reduce_map(zmap, hit_submaps=hits, global2local=g2l)
+                tdist.reduce_map(zmap, hit_submaps=hits, global2local=g2l, nvls=nvls_red)
             else:
                 tdist.reduce_map(zmap)
         host_map.copy_(zmap, non_blocking=True)
@@ -631,7 +638,8 @@ def run_e2e(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples
                     "256-detector blocks from pinned host memory, copy of block b+1 overlapping the kernel on b"}
 
 
-def run_e2e_round_trip(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples, own, scan_map_in):
+def run_e2e_round_trip(args, obs, zmap, hits, g2l, world, stream, packed, total_det_samples, own, scan_map_in,
+                       nvls_red=None):
     """e2e of the round-trip workloads (c3rt, c5m): every step copies the input map and each
     observation's pointing inputs (focal plane, boresight, HWP, flags; the TOD is the scan's
     output and never leaves the device) from pinned host memory, scans and accumulates through
@@ -681,7 +689,7 @@ def run_e2e_round_trip(args, obs, zmap, hits, g2l, world, stream, packed, total_
                 tdist.reduce_scatter_map(zmap, own)
             elif packed:
                 tdist.union_hit_submaps(hits)
-                tdist.reduce_map(zmap, hit_submaps=hits, global2local=g2l)
+                tdist.reduce_map(zmap, hit_submaps=hits, global2local=g2l, nvls=nvls_red)
             else:
                 tdist.reduce_map(zmap)
         host_map.copy_(zmap, non_blocking=True)

@@ -75,6 +75,7 @@ def load():
     L.toast_template_offset_project_signal.argtypes = [I64, P, P, P, P, P, P, U8, P, I64, I64, I64, P]
     L.toast_template_offset_apply_diag_precond.argtypes = [P, P, P, I64, P]
     L.toast_synth_tod.argtypes = [P, P, P, I64, I64, ctypes.c_uint64, ctypes.c_uint64, P]
+    L.toast_map_allreduce_nvls.argtypes = [P, I64, P, I32, I32, P]
     for name in EXPORTED[4:]:
         getattr(L, name).restype = I32
     _lib = L
@@ -422,6 +423,17 @@ def synth_tod(out, sigma, det_ids, seed: int, stream_id: int = 1, stream=None):
           c(sigma, torch.float64, "sigma", shape=(n_det,)), c(det_ids, torch.int64, "det_ids", shape=(n_det,)),
           n_det, n_samp, int(seed) & ((1 << 64) - 1), int(stream_id), stream=stream)
     return out
+
+
+def map_allreduce_nvls(buf: torch.Tensor, mc_ptr: int, pads_dev_ptr: int, rank: int, world: int, stream=None):
+    """toast_map_allreduce_nvls on `buf` (an f64 tensor in symmetric memory whose multicast mapping
+    starts at device address `mc_ptr`; `pads_dev_ptr` the device array of the ranks' signal pads).
+    Every rank's `buf` holds the sum over ranks afterwards (stream order)."""
+    c = _Call("toast_map_allreduce_nvls")
+    c(buf, torch.float64, "buf")
+    c.run(load().toast_map_allreduce_nvls, ctypes.c_void_p(int(mc_ptr)), buf.numel(),
+          ctypes.c_void_p(int(pads_dev_ptr)) if pads_dev_ptr else None, int(rank), int(world), stream=stream)
+    return buf
 
 
 def pointing_to_map_raw(args: tuple):

@@ -825,3 +825,16 @@ extern "C" int toast_template_offset_apply_diag_precond(const double* offset_var
     if (e != cudaSuccess) return cuda_fail(e, "template_offset_apply_diag_precond launch");
     return ok();
 }
+
+extern "C" int toast_map_allreduce_nvls(double* mc, int64_t n, unsigned* const* pads, int rank, int world,
+                                        void* stream) {
+    using namespace toastb200;
+    if (n < 0) return fail(TOAST_EINVAL, "n = %lld < 0", (long long)n);
+    if (world < 1 || rank < 0 || rank >= world)
+        return fail(TOAST_EINVAL, "rank %d / world %d out of range", rank, world);
+    if (n > 0 && !mc) return fail(TOAST_EINVAL, "mc is NULL");
+    if (world > 1 && !pads) return fail(TOAST_EINVAL, "pads is NULL with world > 1");
+    const cudaError_t e = launch_map_allreduce_nvls(mc, n, pads, rank, world, (cudaStream_t)stream);
+    if (e != cudaSuccess) return cuda_fail(e, "map_allreduce_nvls launch");
+    return ok();
+}

@@ -138,5 +138,7 @@ cudaError_t launch_precond(const double* var, const double* in, double* out, int
 unsigned long long* sched_counter(int* err);
 
 int num_sms();
+cudaError_t launch_map_allreduce_nvls(double* mc, int64_t n, unsigned* const* pads, int rank, int world,
+                                      cudaStream_t st);
 
 }  // namespace toastb200

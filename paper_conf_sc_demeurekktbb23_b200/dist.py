@@ -103,23 +103,70 @@ def hit_local_submaps(hit_submaps: torch.Tensor, global2local: torch.Tensor) -> 
 
 
 def reduce_map(zmap: torch.Tensor, group=None, hit_submaps: Optional[torch.Tensor] = None,
-               global2local: Optional[torch.Tensor] = None) -> Tuple[torch.Tensor, int]:
+               global2local: Optional[torch.Tensor] = None, nvls: Optional["NvlsReducer"] = None
+               ) -> Tuple[torch.Tensor, int]:
     """Sum the per-rank partial maps (zmap [n_local_submap][n_pix_submap][nnz]) in place.
 
     With `hit_submaps` (already the union over ranks) only those submaps travel: packed into
-    a contiguous buffer, all-reduced, unpacked.  Returns (zmap, bytes all-reduced)."""
+    a contiguous buffer, all-reduced, unpacked.  With `nvls` the sum runs in the switch through
+    toast_map_allreduce_nvls instead of NCCL.  Returns (zmap, bytes all-reduced)."""
     if not (dist.is_initialized() and dist.get_world_size(group) > 1):
         return zmap, 0
+
+    def allreduce(t):
+        if nvls is not None:
+            nvls.allreduce_(t)
+        else:
+            dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+
     if hit_submaps is None:
-        dist.all_reduce(zmap, op=dist.ReduceOp.SUM, group=group)
+        allreduce(zmap)
         return zmap, zmap.numel() * zmap.element_size()
     if global2local is None:
         global2local = torch.arange(hit_submaps.numel(), device=zmap.device)
     idx = hit_local_submaps(hit_submaps.to(zmap.device), global2local.to(zmap.device))
     packed = zmap.index_select(0, idx)
-    dist.all_reduce(packed, op=dist.ReduceOp.SUM, group=group)
+    allreduce(packed)
     zmap.index_copy_(0, idx, packed)
     return zmap, packed.numel() * packed.element_size()
+
+
+# ----------------------------------------------------------------------------- NVLS map exchange
+# SURVEY 8(f) f3 / 8(e) step 3 done in the switch by our own kernel (toast_map_allreduce_nvls:
+# multimem.ld_reduce / multimem.st over a multicast mapping) instead of NCCL's all_reduce.  The
+# buffer lives in torch symmetric memory, which creates the per-rank mappings, the multicast
+# object and the signal pads (plumbing only); the reduction itself is the library's kernel.
+
+class NvlsReducer:
+    """A symmetric-memory f64 buffer of `numel` elements with a multicast mapping over the
+    group's ranks.  `allreduce_(t)` sums `t` (numel <= capacity) over the ranks in place, through
+    the buffer (or directly, when `t` is a view of `self.buf` starting at its first element).
+    Raises RuntimeError when the GPUs / driver have no multicast (NVLS) support."""
+
+    def __init__(self, numel: int, device, group=None):
+        import torch.distributed._symmetric_memory as symm_mem
+        group = group or dist.group.WORLD
+        self.buf = symm_mem.empty(int(numel), dtype=torch.float64, device=device)
+        self.hdl = symm_mem.rendezvous(self.buf, group.group_name)
+        if not self.hdl.has_multicast_support or not int(self.hdl.multicast_ptr):
+            raise RuntimeError("no multicast (NVLS) mapping on this device / driver / group")
+        self.rank, self.world = int(self.hdl.rank), int(self.hdl.world_size)
+        self.mc_ptr = int(self.hdl.multicast_ptr)
+        self.pads = int(self.hdl.signal_pad_ptrs_dev)
+
+    def allreduce_(self, t: torch.Tensor) -> torch.Tensor:
+        from . import binding
+        n = t.numel()
+        if n > self.buf.numel():
+            raise ValueError(f"{n} elements > the NVLS buffer's {self.buf.numel()}")
+        inplace = t.data_ptr() == self.buf.data_ptr() and t.is_contiguous()
+        view = self.buf[:n]
+        if not inplace:
+            view.copy_(t.reshape(-1))
+        binding.map_allreduce_nvls(view, self.mc_ptr, self.pads, self.rank, self.world)
+        if not inplace:
+            t.copy_(view.view_as(t))
+        return t
 
 
 # ----------------------------------------------------------------------------- sparse map domain

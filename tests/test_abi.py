@@ -93,6 +93,12 @@ def test_validation_rejects_before_any_launch(lib):
             lib, "epsilon")
     _einval(lib.toast_pointing_detector(dummy, dummy, None, dummy, iv_ok.ctypes.data, 1, None, 0, -1, 10, None), lib,
             "n_det")
+    # the NVLS map exchange (f3): sizes, ranks, pads
+    _einval(lib.toast_map_allreduce_nvls(dummy, -1, None, 0, 1, None), lib, "< 0")
+    _einval(lib.toast_map_allreduce_nvls(dummy, 10, dummy, 2, 2, None), lib, "out of range")
+    _einval(lib.toast_map_allreduce_nvls(dummy, 10, dummy, 0, 0, None), lib, "out of range")
+    _einval(lib.toast_map_allreduce_nvls(None, 10, dummy, 0, 1, None), lib, "mc is NULL")
+    _einval(lib.toast_map_allreduce_nvls(dummy, 10, None, 0, 2, None), lib, "pads is NULL")
 
 
 def test_binding_refuses_cpu_tensors():
