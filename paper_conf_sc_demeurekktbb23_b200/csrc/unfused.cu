@@ -222,6 +222,19 @@ __global__ void __launch_bounds__(kChunk, TB_A3_MINB) stokes_weights_kernel(
 #define TB_A4_DT 1  // measured on B200 (C2): 2 rows per CTA row -4 %, 4 rows -40 % (registers)
 #endif
 constexpr int kA4DT = TB_A4_DT;
+#ifndef TB_A4_ORDER
+#define TB_A4_ORDER 1  // measured r02a4c (A4 ms, C2 / C3 / C5): order 0 0.662 / 0.620 / 3.66, order 1 with 8 / 16 / 32 rows
+#endif               // 0.511 / 0.506 / 2.80, 0.496 / 0.487 / 2.79, 0.494 / 0.486 / 2.97
+#ifndef TB_A4_ROWS
+#define TB_A4_ROWS 16
+#endif
+constexpr int kA4Order = TB_A4_ORDER;
+constexpr int kA4Rows = TB_A4_ROWS;
+dim3 grid_a4(const WorkList& wl, int64_t n_det) {
+    if (kA4Order)
+        return dim3((unsigned)((n_det + kA4Rows - 1) / kA4Rows), (unsigned)std::min<int64_t>(wl.n_chunks, 65535), 1);
+    return grid_for(wl, n_det, kA4DT);
+}
 
 template <int NNZ, bool IDX>
 __global__ void __launch_bounds__(kChunk, TB_A4_MINB) build_noise_weighted_kernel(
@@ -233,7 +246,15 @@ __global__ void __launch_bounds__(kChunk, TB_A4_MINB) build_noise_weighted_kerne
     const double* __restrict__ det_scale, const uint8_t* __restrict__ shared_flags, uint8_t shared_flag_mask,
     int64_t n_det, int64_t n_samp) {
     const int lane = threadIdx.x & 31;
-    for (int64_t c = blockIdx.x; c < n_chunks; c += gridDim.x) {
+    // kA4Order 1: blockIdx.x = a block of kA4Rows consecutive detector rows (fastest), blockIdx.y =
+    // chunk, so the CTAs in flight cover the whole focal plane over one short time window (the
+    // map lines they scatter into stay in L2) and each CTA amortises its chunk setup over
+    // kA4Rows rows.  kA4Order 0: blockIdx.x = chunk, blockIdx.y strides the rows.
+    const int64_t c0 = kA4Order ? blockIdx.y : blockIdx.x, cs = kA4Order ? gridDim.y : gridDim.x;
+    const int64_t r0 = kA4Order ? (int64_t)blockIdx.x * kA4Rows : (int64_t)blockIdx.y * kA4DT;
+    const int64_t r1 = kA4Order ? (r0 + kA4Rows < n_det ? r0 + kA4Rows : n_det) : n_det;
+    const int64_t rs = kA4Order ? kA4DT : (int64_t)gridDim.y * kA4DT;
+    for (int64_t c = c0; c < n_chunks; c += cs) {
         const Chunk ch = chunks[c];
         if ((int)(threadIdx.x & ~31u) >= ch.count) continue;
         const bool in = (int)threadIdx.x < ch.count;
@@ -241,7 +262,7 @@ __global__ void __launch_bounds__(kChunk, TB_A4_MINB) build_noise_weighted_kerne
         const bool sflag = in && shared_flags && (__ldg(&shared_flags[s]) & shared_flag_mask);
         // kA4DT detector rows per CTA row: every row's loads are issued before the first row's
         // segmented scan, so each thread keeps kA4DT x 6 loads in flight
-        for (int64_t d0 = (int64_t)blockIdx.y * kA4DT; d0 < n_det; d0 += (int64_t)gridDim.y * kA4DT) {
+        for (int64_t d0 = r0; d0 < r1; d0 += rs) {
             int64_t key[kA4DT];
             double v0[kA4DT], v1[kA4DT], v2[kA4DT];
 #pragma unroll
@@ -279,20 +300,40 @@ __global__ void __launch_bounds__(kChunk, TB_A4_MINB) build_noise_weighted_kerne
 
 // ----------------------------------------------------------------------------- A5
 
+#ifndef TB_A5_ORDER
+#define TB_A5_ORDER 0  // measured r02a5 (A5 ms, C2 / C3 / C5): order 0 0.538 / 0.520 / 2.98, order 1 (16 rows)
+#endif                 // 0.586 / 0.565 / 2.74: the gathers prefer the chunk-fastest order below nside 4096
+#ifndef TB_A5_ROWS
+#define TB_A5_ROWS 16
+#endif
+constexpr int kA5Order = TB_A5_ORDER;
+constexpr int kA5Rows = TB_A5_ROWS;
+dim3 grid_a5(const WorkList& wl, int64_t n_det) {
+    if (kA5Order)
+        return dim3((unsigned)((n_det + kA5Rows - 1) / kA5Rows), (unsigned)std::min<int64_t>(wl.n_chunks, 65535), 1);
+    return grid_for(wl, n_det, 1);
+}
+
 template <int NNZ, bool IDX>
 __global__ void __launch_bounds__(kChunk, TB_A5_MINB) scan_map_kernel(
     const Chunk* __restrict__ chunks, int64_t n_chunks, MapGeom mg, const double* __restrict__ mapdata,
     const int32_t* __restrict__ data_index, double* __restrict__ det_data, const int32_t* __restrict__ pixel_index,
     const int64_t* __restrict__ pixels, const int32_t* __restrict__ weight_index, const double* __restrict__ weights,
     double data_scale, int should_zero, int should_subtract, int64_t n_det, int64_t n_samp) {
-    for (int64_t c = blockIdx.x; c < n_chunks; c += gridDim.x) {
+    // kA5Order 1: blockIdx.x = kA5Rows consecutive detector rows (fastest), blockIdx.y = chunk (the
+    // CTAs in flight gather from the map around one short time window of the whole focal plane)
+    const int64_t c0 = kA5Order ? blockIdx.y : blockIdx.x, cs = kA5Order ? gridDim.y : gridDim.x;
+    const int64_t r0 = kA5Order ? (int64_t)blockIdx.x * kA5Rows : (int64_t)blockIdx.y;
+    const int64_t r1 = kA5Order ? (r0 + kA5Rows < n_det ? r0 + kA5Rows : n_det) : n_det;
+    const int64_t rs = kA5Order ? 1 : (int64_t)gridDim.y;
+    for (int64_t c = c0; c < n_chunks; c += cs) {
         const Chunk ch = chunks[c];
         if ((int)threadIdx.x >= ch.count) continue;
         const int64_t s = ch.first + threadIdx.x;
         // one detector per CTA row: the gather's three dependent loads per detector are
         // latency-bound, and more resident CTAs hide them better than batching detectors
         // (measured: 86 % vs 59 % of HBM bandwidth with 4 detectors per CTA)
-        for (int64_t d = blockIdx.y; d < n_det; d += gridDim.y) {
+        for (int64_t d = r0; d < r1; d += rs) {
             const int64_t pix = __ldg(&pixels[row_of<IDX>(pixel_index, d) * n_samp + s]);
             if (pix < 0) continue;
             int64_t sm, lp;
@@ -375,11 +416,11 @@ cudaError_t launch_build_noise_weighted(const WorkList& wl, const MapGeom& mg, d
                                         uint8_t shared_flag_mask, int64_t n_det, int64_t n_samp, cudaStream_t st) {
     if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
     if (nnz == 3)
-        (pixel_index || weight_index || data_index || flag_index ? build_noise_weighted_kernel<3, true> : build_noise_weighted_kernel<3, false>)<<<grid_for(wl, n_det, kA4DT), kChunk, 0, st>>>(
+        (pixel_index || weight_index || data_index || flag_index ? build_noise_weighted_kernel<3, true> : build_noise_weighted_kernel<3, false>)<<<grid_a4(wl, n_det), kChunk, 0, st>>>(
             wl.chunks, wl.n_chunks, mg, zmap, pixel_index, pixels, weight_index, weights, data_index, det_data,
             flag_index, det_flags, det_flag_mask, det_scale, shared_flags, shared_flag_mask, n_det, n_samp);
     else
-        (pixel_index || weight_index || data_index || flag_index ? build_noise_weighted_kernel<1, true> : build_noise_weighted_kernel<1, false>)<<<grid_for(wl, n_det, kA4DT), kChunk, 0, st>>>(
+        (pixel_index || weight_index || data_index || flag_index ? build_noise_weighted_kernel<1, true> : build_noise_weighted_kernel<1, false>)<<<grid_a4(wl, n_det), kChunk, 0, st>>>(
             wl.chunks, wl.n_chunks, mg, zmap, pixel_index, pixels, weight_index, weights, data_index, det_data,
             flag_index, det_flags, det_flag_mask, det_scale, shared_flags, shared_flag_mask, n_det, n_samp);
     return cudaGetLastError();
@@ -392,12 +433,12 @@ cudaError_t launch_scan_map(const WorkList& wl, const MapGeom& mg, const double*
                             cudaStream_t st) {
     if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
     if (nnz == 3)
-        (data_index || pixel_index || weight_index ? scan_map_kernel<3, true> : scan_map_kernel<3, false>)<<<grid_for(wl, n_det, 1), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, mg, mapdata, data_index,
+        (data_index || pixel_index || weight_index ? scan_map_kernel<3, true> : scan_map_kernel<3, false>)<<<grid_a5(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, mg, mapdata, data_index,
                                                                     det_data, pixel_index, pixels, weight_index,
                                                                     weights, data_scale, should_zero,
                                                                     should_subtract, n_det, n_samp);
     else
-        (data_index || pixel_index || weight_index ? scan_map_kernel<1, true> : scan_map_kernel<1, false>)<<<grid_for(wl, n_det, 1), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, mg, mapdata, data_index,
+        (data_index || pixel_index || weight_index ? scan_map_kernel<1, true> : scan_map_kernel<1, false>)<<<grid_a5(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, mg, mapdata, data_index,
                                                                     det_data, pixel_index, pixels, weight_index,
                                                                     weights, data_scale, should_zero,
                                                                     should_subtract, n_det, n_samp);
