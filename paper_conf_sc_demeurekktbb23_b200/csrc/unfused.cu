@@ -73,12 +73,32 @@ constexpr int kA1DT = TB_A1_DT;  // A1: detectors per thread (stores only: no re
 
 // ----------------------------------------------------------------------------- A1
 
+#ifndef TB_A1_ORDER
+#define TB_A1_ORDER 0
+#endif
+#ifndef TB_A1_ROWS
+#define TB_A1_ROWS 16
+#endif
+constexpr int kA1Order = TB_A1_ORDER;
+constexpr int kA1Rows = TB_A1_ROWS;
+dim3 grid_a1(const WorkList& wl, int64_t n_det) {
+    if (kA1Order)
+        return dim3((unsigned)((n_det + kA1Rows - 1) / kA1Rows), (unsigned)std::min<int64_t>(wl.n_chunks, 65535), 1);
+    return grid_for(wl, n_det, kA1DT);
+}
+
 template <bool IDX>
 __global__ void __launch_bounds__(kChunk, TB_A1_MINB) pointing_detector_kernel(
     const Chunk* __restrict__ chunks, int64_t n_chunks, const double* __restrict__ fp_quats,
     const double* __restrict__ boresight, const int32_t* __restrict__ quat_index, double* __restrict__ quats,
     const uint8_t* __restrict__ shared_flags, uint8_t shared_flag_mask, int64_t n_det, int64_t n_samp) {
-    for (int64_t c = blockIdx.x; c < n_chunks; c += gridDim.x) {
+    // kA1Order 1: blockIdx.x = kA1Rows consecutive detector rows (fastest), blockIdx.y = chunk: one
+    // boresight load per thread serves kA1Rows rows of streaming stores
+    const int64_t c0 = kA1Order ? blockIdx.y : blockIdx.x, cs = kA1Order ? gridDim.y : gridDim.x;
+    const int64_t r0 = kA1Order ? (int64_t)blockIdx.x * kA1Rows : (int64_t)blockIdx.y * kA1DT;
+    const int64_t r1 = kA1Order ? (r0 + kA1Rows < n_det ? r0 + kA1Rows : n_det) : n_det;
+    const int64_t rs = kA1Order ? kA1DT : (int64_t)gridDim.y * kA1DT;
+    for (int64_t c = c0; c < n_chunks; c += cs) {
         const Chunk ch = chunks[c];
         if ((int)threadIdx.x >= ch.count) continue;
         const int64_t s = ch.first + threadIdx.x;
@@ -88,11 +108,11 @@ __global__ void __launch_bounds__(kChunk, TB_A1_MINB) pointing_detector_kernel(
         if (shared_flags && (__ldg(&shared_flags[s]) & shared_flag_mask)) {
             b[0] = 0.0; b[1] = 0.0; b[2] = 0.0; b[3] = 1.0;  // reading S2
         }
-        for (int64_t d0 = (int64_t)blockIdx.y * kA1DT; d0 < n_det; d0 += (int64_t)gridDim.y * kA1DT) {
+        for (int64_t d0 = r0; d0 < r1; d0 += rs) {
 #pragma unroll
             for (int j = 0; j < kA1DT; ++j) {
                 const int64_t d = d0 + j;
-                if (d >= n_det) break;
+                if (d >= r1) break;
                 double f[4], q[4];
                 load_quat(fp_quats + 4 * d, f);
                 quat_mul(b, f, q);
@@ -369,7 +389,7 @@ cudaError_t launch_pointing_detector(const WorkList& wl, const double* fp_quats,
                                      const int32_t* quat_index, double* quats, const uint8_t* shared_flags,
                                      uint8_t shared_flag_mask, int64_t n_det, int64_t n_samp, cudaStream_t st) {
     if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
-    (quat_index ? pointing_detector_kernel<true> : pointing_detector_kernel<false>)<<<grid_for(wl, n_det, kA1DT), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, fp_quats, boresight,
+    (quat_index ? pointing_detector_kernel<true> : pointing_detector_kernel<false>)<<<grid_a1(wl, n_det), kChunk, 0, st>>>(wl.chunks, wl.n_chunks, fp_quats, boresight,
                                                                       quat_index, quats, shared_flags,
                                                                       shared_flag_mask, n_det, n_samp);
     return cudaGetLastError();
