@@ -186,6 +186,15 @@ __global__ void __launch_bounds__(kChunk) offset_project_kernel(
 // (Measured alternative: coalesced loads staged through a padded shared-memory transpose, 1.7x
 // slower.)
 constexpr int kSpan = 8;
+// measured r02pj (project ms, C2 / C3 / C5): scalar loads, 1 row per warp 0.193 / 0.173 / 0.662 (44-50 %
+// of HBM); 16-byte loads 0.126 / 0.116 / 0.481; 4 rows per warp 0.161 / 0.153 / 0.586; both 0.109 /
+// 0.101 / 0.387 (79-85 %)
+#ifndef TB_PROJ_VEC
+#define TB_PROJ_VEC 1
+#endif
+#ifndef TB_PROJ_ROWS
+#define TB_PROJ_ROWS 4
+#endif
 static_assert(kSpan * 32 == kChunk, "a warp covers one work chunk");
 
 template <bool IDX>
@@ -218,6 +227,26 @@ __global__ void __launch_bounds__(kChunk) offset_project_span_kernel(
             const double* t = det_data + row_or<IDX>(data_index, d) * n_samp + s0;
             const uint8_t* f = det_flags ? det_flags + row_or<IDX>(flag_index, d) * n_samp + s0 : nullptr;
             double A = 0.0, B = 0.0;
+#if TB_PROJ_VEC
+            // the lane's 8 samples as 4 x 16-byte loads (and its 8 flag bytes as one) when aligned
+            if (n == kSpan && ((reinterpret_cast<uintptr_t>(t) & 15u) == 0) &&
+                (!f || (reinterpret_cast<uintptr_t>(f) & 7u) == 0)) {
+                double xv[kSpan];
+#pragma unroll
+                for (int k = 0; k < kSpan; k += 2) {
+                    const double2 q = __ldg(reinterpret_cast<const double2*>(t + k));
+                    xv[k] = q.x;
+                    xv[k + 1] = q.y;
+                }
+                unsigned long long fb = 0ull;
+                if (f) fb = __ldg(reinterpret_cast<const unsigned long long*>(f));
+#pragma unroll
+                for (int k = 0; k < kSpan; ++k) {
+                    const double x = ((fb >> (8 * k)) & det_flag_mask) ? 0.0 : xv[k];
+                    if (k < kb) A += x; else B += x;
+                }
+            } else
+#endif
 #pragma unroll
             for (int k = 0; k < kSpan; ++k) {
                 if (k < n) {
@@ -282,8 +311,11 @@ cudaError_t launch_offset_project(const WorkList& wl, const OffsetViews& v, cons
     if (wl.n_chunks == 0 || n_det == 0) return cudaSuccess;
     const bool idx = data_index || flag_index;
     if (v.step >= kSpan) {
+        // TB_PROJ_ROWS detector rows per warp (the y-stride loop), so each warp amortises its
+        // chunk's step bookkeeping over several rows
+        const int64_t rows = (int64_t)(kChunk / 32) * TB_PROJ_ROWS;
         const dim3 grid((unsigned)std::min<int64_t>(wl.n_chunks, 0x7fffffff),
-                        (unsigned)std::min<int64_t>((n_det + kChunk / 32 - 1) / (kChunk / 32), 65535), 1);
+                        (unsigned)std::min<int64_t>((n_det + rows - 1) / rows, 65535), 1);
         (idx ? offset_project_span_kernel<true> : offset_project_span_kernel<false>)<<<grid, kChunk, 0, st>>>(
             wl.chunks, wl.n_chunks, v, amp_offset, amplitudes, data_index, det_data, flag_index, det_flags,
             det_flag_mask, n_det, n_samp);
