@@ -29,6 +29,10 @@
 //     shared-memory cache, one fp64 `red` per Stokes component (measured against a converged
 //     per-warp flush queue: the queue won 2 % at C2 and lost 8-10 % at C3/C5, where some lane of
 //     the 32 changes pixel at most samples anyway).
+//   * PIPE kernels (the production map direction): the run that ended at sample k is flushed at
+//     sample k+1 as straight-line predicated code in the same basic block as k+1's pointing, so
+//     its integer decode / lookup / reduction chain interleaves with independent fp64 work
+//     (nside >= 1024: always; below: the hybrid form, only when some lane has a pending run).
 //   * SCAN mode gathers the map instead (cached per lane across the run) and updates the
 //     staged TOD, written back after each half block.
 #include <cuda.h>  // CUtensorMap (the encoder is fetched through the runtime; no -lcuda)
