@@ -953,6 +953,73 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
                     }
                 }
             }
+            if constexpr (SCAN && PIPE != 0 && !WIDE) {
+                if (scan_lean) {
+                    // PIPE scan: straight-line per sample (predicated shared / global accesses), so
+                    // the run's decode -> lookup -> gather chain interleaves with the next sample's
+                    // pointing in the unrolled loop; a lane whose key did not change keeps its run
+                    piped = true;
+                    const int kb = cur.k0, ke = cur.k0 + cur.nb;
+                    const unsigned psm_mask = (unsigned)(mg.n_pix_submap - 1);
+                    const unsigned pm = sl.ok ? pmask : 0u;
+                    const int okm = sl.ok ? 0 : -1;
+                    const double sgn = sgn_ds;
+#pragma unroll kPipeUnroll
+                    for (int k = kb; k < ke; ++k) {
+                        const unsigned addr = tile ^ ((unsigned)k << 3);
+                        double x[12];
+                        load_state(k, x);
+                        {  // the pending update of the previous sample (t = data_scale sum_k m_k w_k)
+                            const unsigned pa = sl.pend_addr;
+                            const unsigned go = pa != 0xffffffffu;
+                            double t = sl.r0 * a.cal;
+                            if (NNZ == 3) t = fma(sl.r1, sl.pend_c, fma(sl.r2, sl.pend_s, t));
+                            double old = 0.0;
+                            if (!a.should_zero)
+                                asm("{\n .reg .pred q;\n setp.ne.u32 q, %1, 0;\n @q ld.shared.f64 %0, [%2];\n}\n"
+                                    : "+d"(old)
+                                    : "r"(go), "r"(pa));
+                            const double v = fma(sgn, t, old);
+                            asm volatile("{\n .reg .pred q;\n setp.ne.u32 q, %0, 0;\n @q st.shared.f64 [%1], %2;\n}\n" ::"r"(go),
+                                         "r"(pa), "d"(v)
+                                         : "memory");
+                        }
+                        const StageA o = stage_a<NNZ, HWP, P>(sl, x, kc);
+                        int key;
+                        if constexpr (HWP && NNZ == 3)
+                            key = (int)stage_b<NEST, NNZ, WIDE>(o, (pm >> k) & 1u, g, kc);
+                        else
+                            key = (int)stage_b<NEST, NNZ, WIDE>(o, true, g, kc) | __double2loint(x[9]) | okm;
+                        const bool valid = key >= 0;
+                        const bool chg = valid && key != (int)sl.run_key;
+                        const unsigned pix = (unsigned)ckey_to_pix_bf<NEST, OFF>(chg ? key : 0, g);
+                        const unsigned loc = cm.g2l[pix >> mg.sm_shift] & 0x7fffu;
+                        const unsigned elem = (loc << mg.sm_shift) + (pix & psm_mask);
+                        const unsigned ld = chg && loc != kNoLoc;
+                        const double* mp = a.mapdata + (size_t)(ld ? elem : 0u) * NNZ;
+                        asm("{\n .reg .pred q;\n setp.ne.u32 q, %1, 0;\n @q ld.global.nc.f64 %0, [%2];\n}\n"
+                            : "+d"(sl.r0)
+                            : "r"(ld), "l"(mp));
+                        if (NNZ == 3) {
+                            asm("{\n .reg .pred q;\n setp.ne.u32 q, %1, 0;\n @q ld.global.nc.f64 %0, [%2];\n}\n"
+                                : "+d"(sl.r1)
+                                : "r"(ld), "l"(mp + 1));
+                            asm("{\n .reg .pred q;\n setp.ne.u32 q, %1, 0;\n @q ld.global.nc.f64 %0, [%2];\n}\n"
+                                : "+d"(sl.r2)
+                                : "r"(ld), "l"(mp + 2));
+                        }
+                        if (chg) {
+                            sl.run_key = key;
+                            sl.run_elem = loc == kNoLoc ? -1 : (int64_t)elem;
+                        }
+                        sl.pend_addr = (valid && sl.run_elem >= 0) ? addr : 0xffffffffu;
+                        if (NNZ == 3) {
+                            sl.pend_c = sl.etacal * (o.cw * o.invr);
+                            sl.pend_s = (2.0 * sl.etacal) * (o.sw * o.invr);
+                        }
+                    }
+                }
+            }
             if (!piped) {
                 const int kb = cur.k0, ke = cur.k0 + cur.nb;
 #pragma unroll 1
@@ -1065,6 +1132,8 @@ __global__ void __launch_bounds__(kWarps * 32, TB_FUSED_MINB)
                         }
                     }
                 }
+            }
+            {
                 scan_finish();  // the block's last pending update, before the write-back
                 __syncwarp();
                 if constexpr (SCAN) {
@@ -1247,6 +1316,9 @@ constexpr int64_t kCompactMaxNside = 4096;
 
 // The pipelined predicated flush (PIPE kernels) for nside >= TB_PIPE_MIN_NSIDE, where some lane of
 // a warp ends a run at nearly every sample anyway.
+#ifndef TB_SCAN_PIPE
+#define TB_SCAN_PIPE 0  // the straight-line (PIPE) scan loop: measured r02sp C3 0.500 -> 0.489 ms, C5 2.704 -> 2.749: off
+#endif
 #ifndef TB_PIPE_HYB
 #define TB_PIPE_HYB 1  // below TB_PIPE_MIN_NSIDE: the hybrid PIPE loop (measured r02p9: C2 0.462 -> 0.451 ms; C3 +3.6 %, C4 +4.3 % with it)
 #endif
@@ -1394,6 +1466,11 @@ cudaError_t dispatch_scan(const WorkList& wl, const FusedArgs& a, unsigned long 
     const bool hwp = a.hwp && NNZ == 3;
     if (wide) return hwp ? launch_t<NEST, NNZ, true, false, true, true>(wl, a, sched, st)
                          : launch_t<NEST, NNZ, false, false, true, true>(wl, a, sched, st);
+#if TB_SCAN_PIPE
+    if (a.nside >= TB_PIPE_MIN_NSIDE)
+        return hwp ? launch_t<NEST, NNZ, true, false, false, true, false, 1>(wl, a, sched, st)
+                   : launch_t<NEST, NNZ, false, false, false, true, false, 1>(wl, a, sched, st);
+#endif
     return hwp ? launch_t<NEST, NNZ, true, false, false, true>(wl, a, sched, st)
                : launch_t<NEST, NNZ, false, false, false, true>(wl, a, sched, st);  // (no queue: a scan gathers)
 }
