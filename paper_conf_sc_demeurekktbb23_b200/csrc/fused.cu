@@ -1385,15 +1385,34 @@ __global__ void __launch_bounds__(256) pointing_to_map_thin_kernel(const Chunk* 
                 add_run<NNZ>(locate(key_to_pixel<NEST, OFF, WIDE>(sl.run_key, g), a, cm), sl.r0 * sl.sI,
                              sl.r1 * sl.sQ, sl.r2 * sl.sU, a, d);
         };
-        for (int64_t s = ch.first; s < ch.first + ch.count; ++s) {
-            if (a.shared_flags && (__ldg(&a.shared_flags[s]) & a.shared_flag_mask)) continue;  // no pixel (S2)
-            const double2 q01 = __ldg(reinterpret_cast<const double2*>(a.boresight + 4 * s));
-            const double2 q23 = __ldg(reinterpret_cast<const double2*>(a.boresight + 4 * s) + 1);
+        // the inputs of sample s+1 are loaded while sample s is computed (one sample ahead): each
+        // thread walks its chunk serially, so without it every sample waits a full DRAM latency
+        struct In {
+            double2 q01, q23;
+            double tod, chi;
+            bool skip;
+        };
+        const int64_t s_end = ch.first + ch.count;
+        auto fetch = [&](int64_t s) {
+            In v;
+            v.skip = a.shared_flags && (__ldg(&a.shared_flags[s]) & a.shared_flag_mask);  // no pixel (S2)
+            v.q01 = __ldg(reinterpret_cast<const double2*>(a.boresight + 4 * s));
+            v.q23 = __ldg(reinterpret_cast<const double2*>(a.boresight + 4 * s) + 1);
+            v.chi = (HWP && NNZ == 3) ? __ldg(&a.hwp[s]) : 0.0;
+            v.tod = __ldg(&a.det_data[d * a.n_samp + s]);
+            if (a.det_flags && (__ldg(&a.det_flags[d * a.n_samp + s]) & a.det_flag_mask)) v.tod = 0.0;
+            return v;
+        };
+        In nx = fetch(ch.first);
+        for (int64_t s = ch.first; s < s_end; ++s) {
+            const In cu = nx;
+            if (s + 1 < s_end) nx = fetch(s + 1);
+            if (cu.skip) continue;
             double x[12];
-            quat_to_matrix(q01.x, q01.y, q23.x, q23.y, x);
+            quat_to_matrix(cu.q01.x, cu.q01.y, cu.q23.x, cu.q23.y, x);
             if (HWP && NNZ == 3) {
                 double s4, c4;
-                const double a4 = 4.0 * __ldg(&a.hwp[s]);
+                const double a4 = 4.0 * cu.chi;
                 if (fabs(a4) < 1.6e6)
                     small_sincos(a4, &s4, &c4);
                 else
@@ -1402,8 +1421,7 @@ __global__ void __launch_bounds__(256) pointing_to_map_thin_kernel(const Chunk* 
                 x[10] = 2.0 * s4;
                 x[11] = 0.5 * s4;
             }
-            double tod = __ldg(&a.det_data[d * a.n_samp + s]);
-            if (a.det_flags && (__ldg(&a.det_flags[d * a.n_samp + s]) & a.det_flag_mask)) tod = 0.0;
+            const double tod = cu.tod;
             const StageA o = stage_a<NNZ, HWP, P>(sl, x, kc);
             const P key = stage_b<NEST, NNZ, WIDE>(o, true, g, kc);
             if (key != sl.run_key) {
