@@ -212,7 +212,10 @@ int fused_worklist(const toast_interval_t* iv, int64_t n, int64_t n_samp, int64_
     // chunks: the warps in flight then span half the time window, so the map lines they scatter
     // into are reused more in L2 (C5 2.57 -> 2.46 ms); at nside 2048 (C4) the longer chunks win
     // (fewer item switches and full-arctangent restarts: C4 46.4 -> 45.6 ms, r02p8)
-    int chunk = (groups >= 64 && nside >= 4096) ? kFusedChunk / 2 : kFusedChunk;
+#ifndef TB_FINE_MAP_CHUNK
+#define TB_FINE_MAP_CHUNK (kFusedChunk / 2)  // C5 (r02fm): 64 2.479 ms, 48 2.498, 32 2.659
+#endif
+    int chunk = (groups >= 64 && nside >= 4096) ? TB_FINE_MAP_CHUNK : kFusedChunk;
     while (chunk > 16 && (n_samples / chunk) * groups < want) chunk /= 2;
 #ifndef TB_NO_TAIL
     const int64_t tail =
